@@ -1,0 +1,274 @@
+/*
+ * rrl.h -- C ABI of the rerooted, level-batched phylogenetic partial-likelihood
+ * library (B200 / sm_100a).  From-scratch implementation of the data-parallel
+ * hot path of Ayres & Cummings, "Rerooting Trees Increases Opportunities for
+ * Concurrent Computation ..." (IPDPSW 2018), cited as PAPER.md:<line> §<sec>.
+ *
+ * Hot path:
+ *   reroot (host) -> schedule (host) -> transition matrices (K1)
+ *   -> one updatePartials launch per level set (K2 4-state / K3 61-state)
+ *   -> scale accumulation (K5, or fused) -> root / edge log-likelihood (K4/K6)
+ *   -> [multi-GPU: all-reduce of the fp64 sum, done by the caller through
+ *       torch.distributed -- not part of this ABI].
+ *
+ * ---------------------------------------------------------------------------
+ * Conventions (apply to every function below)
+ * ---------------------------------------------------------------------------
+ * Return value: int.  >= 0 is success (create returns an instance id, the
+ *   others 0).  < 0 is one of the RRL_ERROR_* codes.  rrl_error_string(code)
+ *   returns static text; rrl_last_error_message() returns a thread-local,
+ *   human-readable description of the last failure (e.g. the CUDA error).
+ * Ownership: every pointer argument is caller-owned.  Host pointers are read
+ *   (or written) only during the call; the library copies inputs and never
+ *   retains caller pointers.  Functions whose name ends in _device take a
+ *   DEVICE pointer on the instance's device, written asynchronously on the
+ *   instance stream.  The instance owns its device memory until
+ *   rrl_finalize_instance.  One instance = one CUDA device + one stream.
+ *   Calls on one instance are not re-entrant; distinct instances may be used
+ *   from distinct threads.
+ * Indices: partials buffers 0..tip_count-1 are the tips (PAPER.md:83:
+ *   n tips, n-1 internal "subtree operations"); buffers tip_count.. are
+ *   internal.  RRL_NONE (-1) means "absent".
+ * Layouts (row-major, host side):
+ *   transition matrix  P[c][z][x] = Pr(child state x | parent state z, r_c t)
+ *                      (Eq. (1) PAPER.md:55 §II-A; reading A2);
+ *   partials (get/set) L[c][p][s]  (category, pattern, state);
+ *   tip states         uint8/int32 [p], 0..s-1, code s (or any value >= s,
+ *                      or < 0) = missing -> all-ones partials (reading A23);
+ *   eigensystem        V[s][s], Vinv[s][s], lambda[s] with
+ *                      Q = V diag(lambda) Vinv.
+ * Device layouts (for readers of DESIGN.md; not part of the ABI):
+ *   4-state partials [p][c][4]; 61-state partials [c][p][64] (padded).
+ * Precision: 32 or 64 (partials, matrices and kernel arithmetic); transition
+ *   matrices are always computed in fp64 and rounded on store; root/edge
+ *   integration always accumulates in fp64.
+ * Errors: invalid arguments return RRL_ERROR_OUT_OF_RANGE (indices) or
+ *   RRL_ERROR_GENERAL without touching state; CUDA failures return
+ *   RRL_ERROR_CUDA.  A non-finite log-likelihood returns
+ *   RRL_ERROR_FLOATING_POINT with the value still written.
+ */
+#ifndef RRL_H
+#define RRL_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RRL_SUCCESS 0
+#define RRL_ERROR_GENERAL (-1)
+#define RRL_ERROR_OUT_OF_MEMORY (-2)
+#define RRL_ERROR_UNIDENTIFIED_EXCEPTION (-3)
+#define RRL_ERROR_UNINITIALIZED_INSTANCE (-4)
+#define RRL_ERROR_OUT_OF_RANGE (-5)
+#define RRL_ERROR_NO_RESOURCE (-6)
+#define RRL_ERROR_NO_IMPLEMENTATION (-7)
+#define RRL_ERROR_FLOATING_POINT (-8)
+#define RRL_ERROR_INVALID_TREE (-9)
+#define RRL_ERROR_CUDA (-10)
+
+#define RRL_NONE (-1)
+
+/* Instance flags (rrl_create_instance). */
+#define RRL_FLAG_SCALE_CUMULATIVE 0x1u /* dest scale = own exponent + children's
+                                          (child scale buffer = child - tip_count);
+                                          no separate accumulation pass needed */
+#define RRL_FLAG_CUDA_GRAPH 0x2u       /* capture each distinct operation list's
+                                          level-set launches in a CUDA graph and
+                                          replay it on later identical calls */
+
+/* Schedule flags (rrl_reroot_and_schedule). Low byte = mode. */
+#define RRL_SCHED_SEQUENTIAL 1u  /* post-order, one op per set (Fig.2 upper) */
+#define RRL_SCHED_LEVEL 2u       /* level sets on the given rooting */
+#define RRL_SCHED_REROOT 3u      /* optimal reroot + level sets */
+#define RRL_SCHED_REUSE_BUFFERS 0x100u /* liveness-based internal buffer reuse */
+
+/* One subtree operation = Eq. (1) for one internal node (PAPER.md:53-55,
+ * Fig. 1):  dest(z) = (sum_x P_matrix1[z][x] child1(x)) *
+ *                     (sum_y P_matrix2[z][y] child2(y))
+ * for every pattern, category and parent state z.
+ * dest_scale_write >= 0: per pattern, m = max over (c, z) of dest; e = the
+ *   frexp exponent of m (m = f 2^e, f in [0.5, 1)); dest *= 2^-e (exact);
+ *   scale buffer dest_scale_write[p] = e  (plus the children's cumulative
+ *   exponents under RRL_FLAG_SCALE_CUMULATIVE)  (reading A5).
+ * dest_scale_read >= 0 (and no write): dest *= 2^-scale[dest_scale_read][p]
+ *   (reuse of existing factors, the paper's rescale-frequency regime A6).
+ * Both RRL_NONE: no rescaling. */
+typedef struct rrl_op {
+  int32_t dest;
+  int32_t dest_scale_write;
+  int32_t dest_scale_read;
+  int32_t child1;
+  int32_t matrix1;
+  int32_t child2;
+  int32_t matrix2;
+} rrl_op;
+
+/* Kernel timing collected when profiling is enabled (CUDA events on the
+ * instance stream around every launch; adds a small gap per launch). */
+typedef struct rrl_profile {
+  double partials_ms;          /* sum of updatePartials set-launch durations */
+  int64_t partials_launches;   /* number of updatePartials launches */
+  double matrices_ms;          /* K1 */
+  int64_t matrices_launches;
+  double root_ms;              /* K4/K6 (+ final reduction) */
+  int64_t root_launches;
+  double scale_ms;             /* K5 */
+  int64_t scale_launches;
+  int64_t kernel_launches;     /* all kernels launched by this instance
+                                  since the last reset (counted always) */
+  int64_t graph_launches;      /* CUDA graph replays (each = many kernels) */
+} rrl_profile;
+
+const char *rrl_error_string(int code);
+const char *rrl_last_error_message(void);
+const char *rrl_version(void);
+
+/* ------------------------------------------------------------------ instance
+ * Create an instance on CUDA device `device` (PAPER.md:167 --rsrc).
+ * tip_count >= 2; partials_buffer_count >= 2*tip_count-1 for a full tree
+ *   (fewer when the caller reuses buffers); state_count in {4, 61}
+ *   (otherwise RRL_ERROR_NO_IMPLEMENTATION); pattern_count >= 1;
+ *   category_count in {1, 2, 4, 8}; precision in {32, 64}.
+ * Returns the instance id (>= 0) or an error. */
+int rrl_create_instance(int tip_count, int partials_buffer_count, int state_count,
+                        int pattern_count, int category_count, int matrix_count,
+                        int eigen_count, int scale_buffer_count, int device,
+                        int precision, uint32_t flags);
+int rrl_finalize_instance(int inst);
+
+/* Use the caller's CUDA stream (e.g. torch.cuda.current_stream().cuda_stream);
+ * NULL restores the instance's own stream. */
+int rrl_set_stream(int inst, void *cuda_stream);
+int rrl_synchronize(int inst);
+
+/* --------------------------------------------------------------------- data
+ * Tip data (reading A23).  Tip partials are category-independent [p][s]. */
+int rrl_set_tip_states(int inst, int tip, const int32_t *states /*[p]*/);
+int rrl_set_tip_states_u8(int inst, int first_tip, int count,
+                          const uint8_t *states /*[count][p]*/);
+int rrl_set_tip_partials(int inst, int tip, const double *partials /*[p][s]*/);
+/* Arbitrary partials for any buffer (tests / restarts), layout [c][p][s]. */
+int rrl_set_partials(int inst, int buffer, const double *partials);
+int rrl_get_partials(int inst, int buffer, double *out /*[c][p][s]*/);
+int rrl_set_pattern_weights(int inst, const double *w /*[p]*/);
+int rrl_set_state_frequencies(int inst, int idx, const double *pi /*[s]*/);
+int rrl_set_category_rates(int inst, const double *r /*[c]*/);
+int rrl_set_category_weights(int inst, int idx, const double *w /*[c]*/);
+
+/* --------------------------------------------------- transition matrices (K1)
+ * P_{m,c} = V diag(exp(lambda * r_c * t_m)) Vinv for each listed matrix m and
+ * every category c, computed in fp64 on the device.  Eq. (1)'s Pr(x|z,t). */
+int rrl_set_eigen_decomposition(int inst, int idx, const double *V, const double *Vinv,
+                                const double *lambda);
+int rrl_update_transition_matrices(int inst, int eigen_idx, const int32_t *matrix_idx,
+                                   const double *t, int count);
+int rrl_set_transition_matrix(int inst, int idx, const double *P /*[c][s][s]*/);
+int rrl_get_transition_matrix(int inst, int idx, double *out /*[c][s][s]*/);
+
+/* ------------------------------------------------------ updatePartials (K2/K3)
+ * Executes `op_count` operations grouped into `set_count` concurrent
+ * operation sets: set k = ops[set_offsets[k] .. set_offsets[k+1]).  Each set
+ * is ONE kernel launch over (pattern-block x operation) (PAPER.md:116, 128
+ * §VI-A "multi-operation kernel"); sets run in order on the instance stream.
+ * Operations inside a set must be mutually independent (no op reads another
+ * op's dest in the same set): violating sets return RRL_ERROR_GENERAL.
+ * set_offsets == NULL: the library batches the ops greedily in submission
+ * order, starting a new set whenever an op depends on an op already in the
+ * current set. */
+int rrl_update_partials(int inst, const rrl_op *ops, int op_count,
+                        const int32_t *set_offsets /*[set_count+1] or NULL*/,
+                        int set_count);
+
+/* ------------------------------------------------------------ scaling (K5)
+ * cumulative[p] += sum_k scale[scale_idx[k]][p]  (int32, exact). */
+int rrl_accumulate_scale_factors(int inst, const int32_t *scale_idx, int count,
+                                 int cumulative_idx);
+int rrl_reset_scale_factors(int inst, int cumulative_idx);
+int rrl_get_scale_factors(int inst, int idx, int32_t *out /*[p]*/);
+
+/* ------------------------------------------------------------- root (K4)
+ * lnL_i = ln( sum_c w_c sum_z pi_z L_root[i][c][z] ) + E_i ln 2,
+ * *out_sum = sum_i wt_i lnL_i (fp64, deterministic fixed-order reduction).
+ * cumulative_idx = RRL_NONE means E = 0.  Blocks until the value is on the
+ * host.  The _device variant writes the fp64 sum to `d_out` (device pointer)
+ * asynchronously; the per-pattern values stay on the device for
+ * rrl_get_site_log_likelihoods. */
+int rrl_calculate_root_log_likelihoods(int inst, int root_buffer, int cat_weights_idx,
+                                       int freqs_idx, int cumulative_idx, double *out_sum);
+int rrl_calculate_root_log_likelihoods_device(int inst, int root_buffer, int cat_weights_idx,
+                                              int freqs_idx, int cumulative_idx,
+                                              double *d_out);
+
+/* ------------------------------------------------------------- edge (K6)
+ * lnL_i = ln( sum_c w_c sum_z pi_z Lp[i][c][z] sum_x P_m[c][z][x] Lc[i][c][x] )
+ *         + (Ep_i + Ec_i) ln 2
+ * parent_scale_idx / child_scale_idx: cumulative exponents of each side
+ * (RRL_NONE = 0).  child_buffer may be a tip. */
+int rrl_calculate_edge_log_likelihoods(int inst, int parent_buffer, int child_buffer,
+                                       int matrix_idx, int cat_weights_idx, int freqs_idx,
+                                       int parent_scale_idx, int child_scale_idx,
+                                       double *out_sum);
+int rrl_get_site_log_likelihoods(int inst, double *out /*[p]*/);
+
+/* ------------------------------------------------------------- profiling */
+int rrl_set_profiling(int inst, int enable);
+int rrl_get_profile(int inst, rrl_profile *out); /* synchronizes the stream */
+int rrl_reset_profile(int inst);
+
+/* ------------------------------------------------ host-only (no instance)
+ * Reroot and schedule (readings A7-A11).
+ * Input: tip_count n >= 2, parent[2n-1] (root = -1; tips 0..n-1, internal
+ * n..2n-2, each internal node with exactly two children), blen[2n-1].
+ * Modes: RRL_SCHED_SEQUENTIAL | LEVEL | REROOT, optionally
+ * | RRL_SCHED_REUSE_BUFFERS.
+ * REROOT picks, in O(n), the unrooted edge minimising the number of level
+ * sets (= tree height), ties broken by (keep current root edge, min
+ * |tips_left - tips_right|, min edge key; edge key = child id in the input
+ * rooting, the root's merged edge = min of its two children), places the new
+ * root (reusing the old root id) at the edge midpoint and merges the old
+ * root's two branches (t1 + t2).
+ * Outputs (caller-allocated):
+ *   out_parent[2n-1], out_blen[2n-1]  -- the (re)rooted tree;
+ *   out_root_edge                      -- key of the root edge chosen;
+ *   out_ops[n-1]                       -- ops, set by set, sorted by dest id,
+ *                                         child1 < child2, matrix = child id,
+ *                                         dest_scale_write = dest - n;
+ *   out_set_offsets[n]                 -- set k = [off[k], off[k+1]);
+ *   out_set_count                      -- number of sets (= height);
+ *   out_buffer_count                   -- partials buffers needed (2n-1, or
+ *                                         fewer with REUSE_BUFFERS, in which
+ *                                         case dest/child/scale ids refer to
+ *                                         physical buffers and out_parent
+ *                                         still uses logical node ids).
+ * Any output pointer may be NULL.  Returns RRL_ERROR_INVALID_TREE for a
+ * malformed tree. */
+int rrl_reroot_and_schedule(int tip_count, const int32_t *parent, const double *blen,
+                            uint32_t flags, int32_t *out_parent, double *out_blen,
+                            int32_t *out_root_edge, rrl_op *out_ops,
+                            int32_t *out_set_offsets, int32_t *out_set_count,
+                            int32_t *out_buffer_count);
+
+/* Per-edge objective table used by the reroot (for tests/reporting):
+ * for each of the 2n-3 unrooted edges, out_key[e], out_sets[e], out_imbalance[e].
+ * Returns the number of edges written. */
+int rrl_reroot_edge_table(int tip_count, const int32_t *parent, int32_t *out_key,
+                          int32_t *out_sets, int32_t *out_imbalance);
+
+/* Substitution model (host, fp64): builds the normalised rate matrix Q
+ * (-sum_i pi_i Q_ii = 1) for model in {"jc69","hky","gtr","gy94"} and its
+ * eigensystem through the symmetric form S = Pi^1/2 Q Pi^-1/2 (cyclic Jacobi).
+ * params: hky {kappa}; gtr {rAC,rAG,rAT,rCG,rCT,rGT}; gy94 {kappa, omega};
+ * jc69 none.  pi[s] must be positive.  Outputs (any may be NULL):
+ * Q[s][s], V[s][s], Vinv[s][s], lambda[s].  s = 4, or 61 for gy94 (sense
+ * codons of the standard code in ACGT order). */
+int rrl_model_eigensystem(const char *model, int state_count, const double *pi,
+                          const double *params, int param_count, double *Q, double *V,
+                          double *Vinv, double *lambda);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RRL_H */

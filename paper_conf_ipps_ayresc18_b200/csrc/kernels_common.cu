@@ -1,0 +1,223 @@
+// K1 transition matrices, K4 root integration, K5 scale accumulation and
+// K6 edge integration (sm_100a).
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "rrl_internal.h"
+
+namespace rrl {
+namespace {
+
+constexpr double kLn2 = 0.693147180559945309417232121458176568;
+
+// ---------------------------------------------------------------------- K1
+// P_{m,c}[z][x] = sum_k V[z][k] exp(lambda_k r_c t_m) Vinv[k][x]  (fp64),
+// Eq. (1)'s Pr(x | z, t) for a reversible Q = V diag(lambda) Vinv.  One block
+// per (listed matrix, category); stored in the instance precision, padded to
+// s_pad x s_pad (padding stays zero).
+template <typename T>
+__global__ void k_transition(int s, int s_pad, int C, const double *__restrict__ eig,
+                             const double *__restrict__ rates, const int32_t *__restrict__ idx,
+                             const double *__restrict__ tlen, T *__restrict__ P) {
+  extern __shared__ double sm[];
+  double *V = sm;
+  double *Vi = sm + s * s;
+  double *ex = sm + 2 * s * s;
+  const int m = blockIdx.x, c = blockIdx.y;
+  const double *lam = eig + 2 * s * s;
+  for (int i = threadIdx.x; i < s * s; i += blockDim.x) {
+    V[i] = eig[i];
+    Vi[i] = eig[s * s + i];
+  }
+  const double rt = rates[c] * tlen[m];
+  for (int k = threadIdx.x; k < s; k += blockDim.x) ex[k] = exp(lam[k] * rt);
+  __syncthreads();
+  T *out = P + ((size_t)idx[m] * C + c) * (size_t)s_pad * s_pad;
+  for (int e = threadIdx.x; e < s * s; e += blockDim.x) {
+    const int z = e / s, x = e % s;
+    double acc = 0.0;
+    for (int k = 0; k < s; ++k) acc = fma(V[z * s + k] * ex[k], Vi[k * s + x], acc);
+    out[z * s_pad + x] = (T)acc;
+  }
+}
+
+// ---------------------------------------------------------------------- K5
+__global__ void k_accumulate(const int32_t *__restrict__ scale, int p_pad,
+                             const int32_t *__restrict__ idx, int count, int32_t *__restrict__ cum,
+                             int p) {
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < p; i += gridDim.x * blockDim.x) {
+    int acc = cum[i];
+    for (int k = 0; k < count; ++k) acc += __ldg(scale + (size_t)__ldg(idx + k) * p_pad + i);
+    cum[i] = acc;
+  }
+}
+
+// Fixed-order block reduction (deterministic for a fixed grid).
+__device__ double block_sum(double v, double *red) {
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  const int w = threadIdx.x >> 5, l = threadIdx.x & 31;
+  if (l == 0) red[w] = v;
+  __syncthreads();
+  double r = 0.0;
+  if (w == 0) {
+    r = (l < (int)(blockDim.x >> 5)) ? red[l] : 0.0;
+    for (int o = 16; o > 0; o >>= 1) r += __shfl_xor_sync(0xffffffffu, r, o);
+  }
+  return r;  // valid in thread 0
+}
+
+template <typename T>
+__device__ inline double site_root(const T *L, int s, int s_pad, int C, int i, int p_pad,
+                                   const double *w, const double *pi) {
+  double acc = 0.0;
+  for (int c = 0; c < C; ++c) {
+    const T *row = (s == 4) ? (L + ((size_t)i * C + c) * 4) : (L + ((size_t)c * p_pad + i) * s_pad);
+    double sc = 0.0;
+    for (int z = 0; z < s; ++z) sc = fma(pi[z], (double)row[z], sc);
+    acc = fma(w[c], sc, acc);
+  }
+  return acc;
+}
+
+// ---------------------------------------------------------------------- K4
+// lnL_i = ln(sum_c w_c sum_z pi_z L_root[i][c][z]) + E_i ln 2; block sums of
+// wt_i lnL_i go to `blocks`, k_final adds them in a fixed order.
+template <typename T>
+__global__ void __launch_bounds__(256)
+k_root(const T *__restrict__ L, int s, int s_pad, int C, const double *__restrict__ w,
+       const double *__restrict__ pi, const int32_t *__restrict__ cum,
+       const double *__restrict__ pw, int p, int p_pad, double *__restrict__ site,
+       double *__restrict__ blocks) {
+  __shared__ double red[32];
+  double part = 0.0;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < p; i += gridDim.x * blockDim.x) {
+    const double a = site_root(L, s, s_pad, C, i, p_pad, w, pi);
+    double l = log(a);
+    if (cum != nullptr) l += (double)cum[i] * kLn2;
+    site[i] = l;
+    part += pw[i] * l;
+  }
+  const double r = block_sum(part, red);
+  if (threadIdx.x == 0) blocks[blockIdx.x] = r;
+}
+
+__global__ void k_final(const double *__restrict__ blocks, int nb, double *__restrict__ out) {
+  __shared__ double red[32];
+  double v = 0.0;
+  for (int i = threadIdx.x; i < nb; i += blockDim.x) v += blocks[i];
+  const double r = block_sum(v, red);
+  if (threadIdx.x == 0) *out = r;
+}
+
+// ---------------------------------------------------------------------- K6
+template <typename T>
+__global__ void __launch_bounds__(256)
+k_edge(const T *__restrict__ Lp, const void *__restrict__ child, int child_is_tip,
+       const T *__restrict__ P, int s, int s_pad, int C, const double *__restrict__ w,
+       const double *__restrict__ pi, const int32_t *__restrict__ cum_p,
+       const int32_t *__restrict__ cum_c, const double *__restrict__ pw, int p, int p_pad,
+       double *__restrict__ site, double *__restrict__ blocks) {
+  __shared__ double red[32];
+  double part = 0.0;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < p; i += gridDim.x * blockDim.x) {
+    double acc = 0.0;
+    const unsigned st = child_is_tip ? (unsigned)static_cast<const uint8_t *>(child)[i] : 0u;
+    for (int c = 0; c < C; ++c) {
+      const size_t off = (s == 4) ? ((size_t)i * C + c) * 4 : ((size_t)c * p_pad + i) * s_pad;
+      const T *lp = Lp + off;
+      const T *lc = child_is_tip ? nullptr : static_cast<const T *>(child) + off;
+      const T *Pc = P + (size_t)c * s_pad * s_pad;
+      double sc = 0.0;
+      for (int z = 0; z < s; ++z) {
+        double v = 0.0;
+        if (child_is_tip) {
+          if (st < (unsigned)s) {
+            v = (double)Pc[z * s_pad + st];
+          } else {
+            for (int x = 0; x < s; ++x) v += (double)Pc[z * s_pad + x];
+          }
+        } else {
+          for (int x = 0; x < s; ++x) v = fma((double)Pc[z * s_pad + x], (double)lc[x], v);
+        }
+        sc = fma(pi[z] * (double)lp[z], v, sc);
+      }
+      acc = fma(w[c], sc, acc);
+    }
+    double l = log(acc);
+    if (cum_p != nullptr) l += (double)cum_p[i] * kLn2;
+    if (cum_c != nullptr) l += (double)cum_c[i] * kLn2;
+    site[i] = l;
+    part += pw[i] * l;
+  }
+  const double r = block_sum(part, red);
+  if (threadIdx.x == 0) blocks[blockIdx.x] = r;
+}
+
+}  // namespace
+
+int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
+                               const double *d_rates, const int32_t *d_idx, const double *d_t,
+                               int count, void *d_P, void *stream) {
+  if (count <= 0) return 0;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const size_t smem = sizeof(double) * (2 * s * s + s);
+  const int threads = (s <= 4) ? 32 : 256;
+  for (int o = 0; o < count; o += 65535) {
+    const int n = (count - o) < 65535 ? (count - o) : 65535;
+    if (prec == 32) {
+      if (smem > 48 * 1024)
+        cudaFuncSetAttribute(k_transition<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      k_transition<float><<<dim3(n, c), threads, smem, st>>>(s, s_pad, c, d_eig, d_rates, d_idx + o,
+                                                             d_t + o, static_cast<float *>(d_P));
+    } else {
+      if (smem > 48 * 1024)
+        cudaFuncSetAttribute(k_transition<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+      k_transition<double><<<dim3(n, c), threads, smem, st>>>(s, s_pad, c, d_eig, d_rates, d_idx + o,
+                                                              d_t + o, static_cast<double *>(d_P));
+    }
+  }
+  return (int)cudaGetLastError();
+}
+
+int launch_accumulate_scale(const int32_t *d_scale, int p_pad, const int32_t *d_idx, int count,
+                            int32_t *d_cum, int p, void *stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  int blocks = (p + 255) / 256;
+  if (blocks > 148 * 8) blocks = 148 * 8;
+  k_accumulate<<<blocks, 256, 0, st>>>(d_scale, p_pad, d_idx, count, d_cum, p);
+  return (int)cudaGetLastError();
+}
+
+int launch_root_lnl(int prec, int s, int s_pad, int c, const void *root, const double *d_w,
+                    const double *d_pi, const int32_t *cum, const double *d_pw, int p, int p_pad,
+                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (prec == 32)
+    k_root<float><<<nblocks, 256, 0, st>>>(static_cast<const float *>(root), s, s_pad, c, d_w, d_pi,
+                                           cum, d_pw, p, p_pad, d_site, d_block);
+  else
+    k_root<double><<<nblocks, 256, 0, st>>>(static_cast<const double *>(root), s, s_pad, c, d_w, d_pi,
+                                            cum, d_pw, p, p_pad, d_site, d_block);
+  k_final<<<1, 256, 0, st>>>(d_block, nblocks, d_out);
+  return (int)cudaGetLastError();
+}
+
+int launch_edge_lnl(int prec, int s, int s_pad, int c, const void *par, const void *child,
+                    int child_is_tip, const void *P, const double *d_w, const double *d_pi,
+                    const int32_t *cum_p, const int32_t *cum_c, const double *d_pw, int p, int p_pad,
+                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (prec == 32)
+    k_edge<float><<<nblocks, 256, 0, st>>>(static_cast<const float *>(par), child, child_is_tip,
+                                           static_cast<const float *>(P), s, s_pad, c, d_w, d_pi,
+                                           cum_p, cum_c, d_pw, p, p_pad, d_site, d_block);
+  else
+    k_edge<double><<<nblocks, 256, 0, st>>>(static_cast<const double *>(par), child, child_is_tip,
+                                            static_cast<const double *>(P), s, s_pad, c, d_w, d_pi,
+                                            cum_p, cum_c, d_pw, p, p_pad, d_site, d_block);
+  k_final<<<1, 256, 0, st>>>(d_block, nblocks, d_out);
+  return (int)cudaGetLastError();
+}
+
+}  // namespace rrl

@@ -1,0 +1,54 @@
+// Internal declarations shared by the host C++ and the CUDA kernels.
+#pragma once
+
+#include <cstdint>
+#include <string>
+
+#include "rrl.h"
+
+namespace rrl {
+
+// Records a thread-local error message and returns `code`.
+int fail(int code, const std::string &msg);
+
+// Resolved operation descriptor, one per rrl_op, resident in device memory.
+// The multi-operation kernel reads its descriptor by blockIdx.y ("pointer
+// arithmetic to allow different input and output arrays for different
+// execution blocks", §VI-A).
+struct DevOp {
+  const void *in1;          // child 1: partials, or uint8 tip states
+  const void *in2;          // child 2
+  void *out;                // dest partials
+  const void *P1;           // [c][s][s] transition matrices of branch 1
+  const void *P2;           // branch 2
+  int32_t *scale_out;       // own (or cumulative) exponent [p], or null
+  const int32_t *scale_in;  // existing factors to apply [p], or null
+  const int32_t *cum1;      // child 1 cumulative exponent (cumulative mode) or null
+  const int32_t *cum2;      // child 2
+  int32_t flags;            // bit0: child1 is tip states, bit1: child2 is tip states
+  int32_t pad;
+};
+static_assert(sizeof(DevOp) == 80, "DevOp layout");
+
+enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2 };
+
+// ---------------------------------------------------------------- launchers
+// All launchers enqueue on `stream` and return cudaError_t as int.
+int launch_update_partials_nuc(int prec, int c, const DevOp *ops, int nops, int p, int p_pad,
+                               void *stream);
+int launch_update_partials_codon(int prec, int c, const DevOp *ops, int nops, int p, int p_pad,
+                                 void *stream);
+int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
+                               const double *d_rates, const int32_t *d_idx, const double *d_t,
+                               int count, void *d_P, void *stream);
+int launch_accumulate_scale(const int32_t *d_scale, int p_pad, const int32_t *d_idx, int count,
+                            int32_t *d_cum, int p, void *stream);
+int launch_root_lnl(int prec, int s, int s_pad, int c, const void *root, const double *d_w,
+                    const double *d_pi, const int32_t *cum, const double *d_pw, int p, int p_pad,
+                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream);
+int launch_edge_lnl(int prec, int s, int s_pad, int c, const void *par, const void *child,
+                    int child_is_tip, const void *P, const double *d_w, const double *d_pi,
+                    const int32_t *cum_p, const int32_t *cum_c, const double *d_pw, int p, int p_pad,
+                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream);
+
+}  // namespace rrl

@@ -1,0 +1,266 @@
+// Host-side reroot + level-set scheduling (C++, O(n)).
+//
+// Implements rrl_reroot_and_schedule / rrl_reroot_edge_table of include/rrl.h.
+// The paper finds the optimal rooting by exhaustive search over every branch
+// (§VI-E, O(n^2)) and notes "a more efficient algorithm could be
+// employed" (§VIII).  This file is that algorithm: the number of
+// concurrent operation sets of a rooting equals its height (BEAGLE's greedy
+// batching of PAPER.md:128 breaks exactly once per dependency level; DESIGN.md
+// reading A7), so one down pass (subtree heights) and one up pass (height of
+// the complementary component) give the set count of every one of the 2n-3
+// candidate root edges in O(n).  Tie-break and rebuild rules: DESIGN.md
+// readings A9-A11.
+#include <algorithm>
+#include <cstdint>
+#include <cstdlib>
+#include <queue>
+#include <vector>
+
+#include "rrl.h"
+#include "rrl_internal.h"
+
+namespace {
+
+struct View {
+  int n = 0, N = 0, root = -1;
+  std::vector<int> parent, c1, c2;  // c1 < c2, -1 for tips
+  std::vector<int> post;            // internal nodes, children before parents
+};
+
+int build_view(int n, const int32_t *parent, View &v) {
+  if (n < 2 || parent == nullptr) return rrl::fail(RRL_ERROR_INVALID_TREE, "need tip_count >= 2");
+  const int N = 2 * n - 1;
+  v.n = n;
+  v.N = N;
+  v.parent.assign(parent, parent + N);
+  v.c1.assign(N, -1);
+  v.c2.assign(N, -1);
+  int roots = 0;
+  for (int x = 0; x < N; ++x) {
+    const int p = parent[x];
+    if (p == -1) {
+      ++roots;
+      v.root = x;
+      continue;
+    }
+    if (p < 0 || p >= N || p == x || p < n)
+      return rrl::fail(RRL_ERROR_INVALID_TREE, "bad parent id");
+    if (v.c1[p] < 0) v.c1[p] = x;
+    else if (v.c2[p] < 0) v.c2[p] = x;
+    else return rrl::fail(RRL_ERROR_INVALID_TREE, "node with more than two children");
+  }
+  if (roots != 1 || v.root < n) return rrl::fail(RRL_ERROR_INVALID_TREE, "need exactly one internal root");
+  for (int x = n; x < N; ++x) {
+    if (v.c2[x] < 0) return rrl::fail(RRL_ERROR_INVALID_TREE, "internal node without two children");
+    if (v.c1[x] > v.c2[x]) std::swap(v.c1[x], v.c2[x]);
+  }
+  // iterative post-order: child1 subtree, child2 subtree, node
+  v.post.clear();
+  v.post.reserve(n - 1);
+  std::vector<std::pair<int, bool>> st;
+  st.reserve(N);
+  st.push_back({v.root, false});
+  int visited = 0;
+  while (!st.empty()) {
+    auto [x, done] = st.back();
+    st.pop_back();
+    if (x < n) {
+      ++visited;
+      continue;
+    }
+    if (done) {
+      v.post.push_back(x);
+      ++visited;
+    } else {
+      st.push_back({x, true});
+      st.push_back({v.c2[x], false});
+      st.push_back({v.c1[x], false});
+    }
+    if ((int)st.size() > N + 1) return rrl::fail(RRL_ERROR_INVALID_TREE, "cycle");
+  }
+  if (visited != N) return rrl::fail(RRL_ERROR_INVALID_TREE, "tree is not connected");
+  return RRL_SUCCESS;
+}
+
+struct EdgeRow {
+  int sets, not_current, imbalance, key;
+  bool operator<(const EdgeRow &o) const {
+    if (sets != o.sets) return sets < o.sets;
+    if (not_current != o.not_current) return not_current < o.not_current;
+    if (imbalance != o.imbalance) return imbalance < o.imbalance;
+    return key < o.key;
+  }
+};
+
+// All 2n-3 unrooted edges with their set counts (O(n) down/up passes).
+std::vector<EdgeRow> edge_table(const View &v) {
+  const int n = v.n, N = v.N, R = v.root;
+  std::vector<int> down(N, 0), tips(N, 0), up(N, 0);
+  for (int x = 0; x < n; ++x) tips[x] = 1;
+  for (int x : v.post) {
+    down[x] = 1 + std::max(down[v.c1[x]], down[v.c2[x]]);
+    tips[x] = tips[v.c1[x]] + tips[v.c2[x]];
+  }
+  const int a = v.c1[R], b = v.c2[R];
+  // up[x] = height of the component on the far side of edge (parent(x), x),
+  // rooted at the neighbour of x across that edge (root's edges merged).
+  up[a] = down[b];
+  up[b] = down[a];
+  for (auto it = v.post.rbegin(); it != v.post.rend(); ++it) {  // parents first
+    const int u = *it;
+    if (u == R) continue;
+    const int l = v.c1[u], r = v.c2[u];
+    up[l] = 1 + std::max(down[r], up[u]);
+    up[r] = 1 + std::max(down[l], up[u]);
+  }
+  std::vector<EdgeRow> rows;
+  rows.reserve(2 * n - 3);
+  const int cur = std::min(a, b);
+  for (int x = 0; x < N; ++x) {
+    if (x == R || x == a || x == b) continue;
+    const int other = n - tips[x];
+    rows.push_back({1 + std::max(down[x], up[x]), 1, std::abs(tips[x] - other), x});
+  }
+  rows.push_back({1 + std::max(down[a], down[b]), 0, std::abs(tips[a] - tips[b]), cur});
+  std::sort(rows.begin(), rows.end(), [](const EdgeRow &p, const EdgeRow &q) { return p.key < q.key; });
+  return rows;
+}
+
+// Re-root on the edge keyed `key` (reading A10/A11): path reversal from the
+// chosen edge up to the old root; the old root id becomes the new root.
+void reroot(const View &v, const double *blen, int key, std::vector<int> &par,
+            std::vector<double> &bl) {
+  const int R = v.root, a = v.c1[R], b = v.c2[R];
+  par = v.parent;
+  bl.assign(blen, blen + v.N);
+  if (key == std::min(a, b)) return;  // already rooted on this edge: no-op (A9(2), A25)
+  const int x0 = key;
+  std::vector<int> path;  // x0, x1 = parent(x0), ..., xk = root child
+  for (int x = x0; x != R; x = v.parent[x]) path.push_back(x);
+  const int k = (int)path.size() - 1;
+  const int c = path[k];
+  const int d = (c == a) ? b : a;
+  const double half = blen[x0] / 2.0;
+  par[x0] = R;
+  bl[x0] = half;
+  par[path[1]] = R;
+  bl[path[1]] = half;
+  for (int i = 1; i <= k - 1; ++i) {
+    par[path[i + 1]] = path[i];
+    bl[path[i + 1]] = blen[path[i]];
+  }
+  par[d] = c;
+  bl[d] = blen[a] + blen[b];
+  par[R] = -1;
+  bl[R] = 0.0;
+}
+
+}  // namespace
+
+extern "C" int rrl_reroot_edge_table(int tip_count, const int32_t *parent, int32_t *out_key,
+                                     int32_t *out_sets, int32_t *out_imbalance) {
+  View v;
+  int rc = build_view(tip_count, parent, v);
+  if (rc < 0) return rc;
+  auto rows = edge_table(v);
+  for (size_t i = 0; i < rows.size(); ++i) {
+    if (out_key) out_key[i] = rows[i].key;
+    if (out_sets) out_sets[i] = rows[i].sets;
+    if (out_imbalance) out_imbalance[i] = rows[i].imbalance;
+  }
+  return (int)rows.size();
+}
+
+extern "C" int rrl_reroot_and_schedule(int tip_count, const int32_t *parent, const double *blen,
+                                       uint32_t flags, int32_t *out_parent, double *out_blen,
+                                       int32_t *out_root_edge, rrl_op *out_ops,
+                                       int32_t *out_set_offsets, int32_t *out_set_count,
+                                       int32_t *out_buffer_count) {
+  try {
+    if (blen == nullptr) return rrl::fail(RRL_ERROR_GENERAL, "blen is NULL");
+    View v;
+    int rc = build_view(tip_count, parent, v);
+    if (rc < 0) return rc;
+    const int n = v.n, N = v.N;
+    const uint32_t mode = flags & 0xffu;
+    if (mode != RRL_SCHED_SEQUENTIAL && mode != RRL_SCHED_LEVEL && mode != RRL_SCHED_REROOT)
+      return rrl::fail(RRL_ERROR_GENERAL, "unknown schedule mode");
+    const bool reuse = (flags & RRL_SCHED_REUSE_BUFFERS) != 0;
+
+    int key = std::min(v.c1[v.root], v.c2[v.root]);
+    if (mode == RRL_SCHED_REROOT) {
+      auto rows = edge_table(v);
+      key = std::min_element(rows.begin(), rows.end())->key;
+    }
+    std::vector<int> par;
+    std::vector<double> bl;
+    reroot(v, blen, key, par, bl);
+    View w;
+    rc = build_view(n, par.data(), w);
+    if (rc < 0) return rc;
+
+    // Operation order and set boundaries.
+    std::vector<int> order;  // internal node ids in execution order
+    std::vector<int> offs;
+    order.reserve(n - 1);
+    if (mode == RRL_SCHED_SEQUENTIAL) {
+      order = w.post;
+      for (int i = 0; i <= (int)order.size(); ++i) offs.push_back(i);
+    } else {
+      std::vector<int> h(N, 0);
+      for (int x : w.post) h[x] = 1 + std::max(h[w.c1[x]], h[w.c2[x]]);
+      const int H = h[w.root];
+      std::vector<int> count(H + 2, 0);
+      for (int x = n; x < N; ++x) ++count[h[x]];
+      offs.assign(H + 1, 0);
+      for (int k = 1; k <= H; ++k) offs[k] = offs[k - 1] + count[k];
+      std::vector<int> fill(offs.begin(), offs.end());
+      order.assign(n - 1, -1);
+      for (int x = n; x < N; ++x) order[fill[h[x] - 1]++] = x;  // ascending ids within a level
+    }
+    const int nsets = (int)offs.size() - 1;
+
+    // Physical buffer assignment (identity unless reusing).
+    std::vector<int> phys(N);
+    for (int x = 0; x < N; ++x) phys[x] = x;
+    int nbuf = N;
+    if (reuse) {
+      std::priority_queue<int, std::vector<int>, std::greater<int>> freeq;
+      int next = n;
+      for (int k = 0; k < nsets; ++k) {
+        for (int i = offs[k]; i < offs[k + 1]; ++i) {
+          const int x = order[i];
+          if (!freeq.empty()) {
+            phys[x] = freeq.top();
+            freeq.pop();
+          } else {
+            phys[x] = next++;
+          }
+        }
+        for (int i = offs[k]; i < offs[k + 1]; ++i) {
+          const int x = order[i];
+          if (w.c1[x] >= n) freeq.push(phys[w.c1[x]]);
+          if (w.c2[x] >= n) freeq.push(phys[w.c2[x]]);
+        }
+      }
+      nbuf = next;
+    }
+
+    if (out_parent) std::copy(par.begin(), par.end(), out_parent);
+    if (out_blen) std::copy(bl.begin(), bl.end(), out_blen);
+    if (out_root_edge) *out_root_edge = key;
+    if (out_ops) {
+      for (int i = 0; i < n - 1; ++i) {
+        const int x = order[i];
+        const int l = w.c1[x], r = w.c2[x];
+        out_ops[i] = rrl_op{phys[x], phys[x] - n, RRL_NONE, phys[l], l, phys[r], r};
+      }
+    }
+    if (out_set_offsets) std::copy(offs.begin(), offs.end(), out_set_offsets);
+    if (out_set_count) *out_set_count = nsets;
+    if (out_buffer_count) *out_buffer_count = nbuf;
+    return RRL_SUCCESS;
+  } catch (...) {
+    return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_reroot_and_schedule");
+  }
+}

@@ -1,0 +1,140 @@
+"""Host orchestration of one likelihood pass through the C ABI (no arithmetic here).
+
+``TreeLikelihood`` is the public entry point a user calls: it owns one
+instance of the library (one GPU, one stream), loads a model / alignment /
+tree, and runs the hot path of SURVEY.md §8(a):
+
+  a1+a2  rrl_reroot_and_schedule      (C++ host, once per tree)
+  a3     rrl_update_transition_matrices (K1)
+  a4     rrl_update_partials            (one K2/K3 launch per level set)
+  a5     scale accumulation             (fused into a4 by default, or K5)
+  a6     rrl_calculate_root_log_likelihoods(_device) (K4)
+  a7     all-reduce of the fp64 sum      (torch.distributed, see parallel.py)
+
+Every numeric step runs in librrl.so; this module only marshals arguments.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import rrl as R
+
+
+def model_param_vector(name: str, kappa: float = 1.0, omega: float = 1.0, exch=None) -> list[float]:
+    if name == "jc69":
+        return []
+    if name == "hky":
+        return [float(kappa)]
+    if name == "gtr":
+        return [float(x) for x in exch]
+    if name == "gy94":
+        return [float(kappa), float(omega)]
+    raise ValueError(name)
+
+
+class TreeLikelihood:
+    """One instance: n tips, p patterns, s states, c categories, fp32|fp64."""
+
+    def __init__(self, n: int, p: int, s: int, c: int, precision: int = 32, device: int = 0,
+                 cumulative_scaling: bool = True, cuda_graph: bool = False,
+                 buffer_count: int | None = None, stream_ptr: int | None = None):
+        self.n, self.p, self.s, self.c, self.precision = n, p, s, c, precision
+        self.cumulative = cumulative_scaling
+        nbuf = buffer_count if buffer_count is not None else 2 * n - 1
+        n_scale = nbuf - n + (0 if cumulative_scaling else 1)
+        flags = (R.FLAG_SCALE_CUMULATIVE if cumulative_scaling else 0) | \
+                (R.FLAG_CUDA_GRAPH if cuda_graph else 0)
+        self.nbuf = nbuf
+        self.n_scale = n_scale
+        self.inst = R.rrl_create_instance(n, nbuf, s, p, c, 2 * n - 1, 1, n_scale, device,
+                                          precision, flags)
+        if stream_ptr is not None:
+            R.rrl_set_stream(self.inst, stream_ptr)
+        self.sched = None
+
+    # ---------------------------------------------------------------- inputs
+    def set_model(self, name: str, pi, rates, cat_weights, kappa=1.0, omega=1.0, exch=None):
+        prm = model_param_vector(name, kappa, omega, exch)
+        Q, V, Vi, lam = R.rrl_model_eigensystem(name, pi, prm)
+        R.rrl_set_eigen_decomposition(self.inst, 0, V, Vi, lam)
+        R.rrl_set_state_frequencies(self.inst, 0, pi)
+        R.rrl_set_category_rates(self.inst, rates)
+        R.rrl_set_category_weights(self.inst, 0, cat_weights)
+        self.Q = Q
+        return Q
+
+    def set_model_params(self, mp, rates, cat_weights):
+        """Convenience for any object with name/pi/kappa/omega/exch attributes."""
+        return self.set_model(mp.name, mp.pi, rates, cat_weights, getattr(mp, "kappa", 1.0),
+                              getattr(mp, "omega", 1.0), getattr(mp, "exch", None))
+
+    def set_tips(self, tips_u8: np.ndarray):
+        R.rrl_set_tip_states_u8(self.inst, 0, tips_u8)
+
+    def set_pattern_weights(self, w):
+        R.rrl_set_pattern_weights(self.inst, w)
+
+    def set_tree(self, parent, blen, mode: str = "reroot", reuse_buffers: bool = False):
+        sch = R.rrl_reroot_and_schedule(self.n, parent, blen, mode, reuse_buffers)
+        if sch["buffer_count"] > self.nbuf:
+            raise ValueError(f"schedule needs {sch['buffer_count']} buffers, instance has {self.nbuf}")
+        par = sch["parent"]
+        self.root = int(np.flatnonzero(par < 0)[0])
+        nonroot = np.flatnonzero(par >= 0).astype(np.int32)
+        self.matrix_idx = nonroot
+        self.t = sch["blen"][nonroot].copy()
+        ops = sch["ops"]
+        # physical buffer holding the root (last op of the last set)
+        self.root_buffer = int(ops["dest"][-1])
+        if not self.cumulative:
+            ops = ops.copy()
+        self.sched = sch
+        self.ops = ops
+        self.offsets = sch["set_offsets"]
+        return sch
+
+    # ---------------------------------------------------------------- pass
+    def update(self):
+        """K1 + all level-set launches (+ K5 when not cumulative)."""
+        R.rrl_update_transition_matrices(self.inst, 0, self.matrix_idx, self.t)
+        R.rrl_update_partials(self.inst, self.ops, self.offsets)
+        if not self.cumulative:
+            cum = self.n_scale - 1
+            R.rrl_reset_scale_factors(self.inst, cum)
+            R.rrl_accumulate_scale_factors(self.inst, self.ops["dest_scale_write"], cum)
+
+    @property
+    def cumulative_idx(self) -> int:
+        return (self.root_buffer - self.n) if self.cumulative else self.n_scale - 1
+
+    def root_loglik(self) -> float:
+        return R.rrl_calculate_root_log_likelihoods(self.inst, self.root_buffer, 0, 0,
+                                                    self.cumulative_idx)
+
+    def root_loglik_device(self, d_out_ptr: int):
+        R.rrl_calculate_root_log_likelihoods_device(self.inst, self.root_buffer, 0, 0,
+                                                    self.cumulative_idx, d_out_ptr)
+
+    def loglik(self) -> float:
+        self.update()
+        return self.root_loglik()
+
+    def site_logliks(self) -> np.ndarray:
+        return R.rrl_get_site_log_likelihoods(self.inst, self.p)
+
+    def partials(self, buffer: int) -> np.ndarray:
+        return R.rrl_get_partials(self.inst, buffer, self.c, self.p, self.s)
+
+    def scale(self, idx: int) -> np.ndarray:
+        return R.rrl_get_scale_factors(self.inst, idx, self.p)
+
+    def close(self):
+        if getattr(self, "inst", None) is not None:
+            R.rrl_finalize_instance(self.inst)
+            self.inst = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass

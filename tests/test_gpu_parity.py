@@ -1,0 +1,254 @@
+"""GPU parity: the CUDA path (through the C ABI) against the fp64 oracle.
+
+Tolerances (BASELINE.json north_star): reroot schedules bit-exact (CPU tests);
+lnL fp64 relative <= 1e-10, fp32 relative <= 1e-4; per-node partials fp32
+<= 1e-5 relative after scaling (per pattern, max over (c, z), reading A19),
+fp64 <= 1e-12.
+"""
+import math
+
+import numpy as np
+import pytest
+
+from oracle import model as om, pruning, reroot as orr
+from workloads import Tree, config_workload, make_workload, with_blen
+
+from ._util import gpu_setup, node_partial_error, oracle_run, rel, rooted
+
+pytestmark = pytest.mark.gpu
+
+LNL_TOL = {64: 1e-10, 32: 1e-4}
+NODE_TOL = {64: 1e-12, 32: 1e-5}
+
+
+@pytest.fixture(scope="module", autouse=True)
+def _built():
+    from paper_conf_ipps_ayresc18_b200 import build
+    build.build()
+
+
+# ------------------------------------------------------------------ K1
+@pytest.mark.parametrize("precision", [64, 32])
+@pytest.mark.parametrize("model", ["jc69", "hky", "gtr"])
+def test_transition_matrices_vs_expm(precision, model):
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="random", n=40, p=10, model=model, c=4, seed=3)
+    tl = gpu_setup(w, "level", precision)
+    tl.update()
+    Q = om.rate_matrix(w.model)
+    tol = 2e-14 if precision == 64 else 2e-7
+    for m in tl.matrix_idx[:20]:
+        got = R.rrl_get_transition_matrix(tl.inst, int(m), w.c, w.s)
+        for k in range(w.c):
+            exp = pruning.transition_matrix(Q, w.rates[k] * w.tree.blen[m])
+            np.testing.assert_allclose(got[k], exp, atol=tol, rtol=0)
+    tl.close()
+
+
+# ------------------------------------------------------------------ lnL parity, configs
+CASES = [
+    ("c0_jc", 64, {}),
+    ("c0_hky", 64, {}),
+    ("c1", 64, {}),
+    ("c1", 32, {}),
+    ("c2", 32, dict(p=20_000)),
+    ("c2", 64, dict(p=20_000)),
+    ("c2_paper", 32, dict(p=5_000)),
+]
+
+
+@pytest.mark.parametrize("name,precision,over", CASES)
+@pytest.mark.parametrize("mode", ["reroot", "level"])
+def test_loglik_matches_oracle(name, precision, over, mode):
+    w = config_workload(name, seed=1, **over)
+    tl = gpu_setup(w, mode, precision)
+    got = tl.loglik()
+    ora = oracle_run(w)                       # ORIGINAL rooting: reroot invariance
+    assert rel(got, ora.lnl) <= LNL_TOL[precision], (got, ora.lnl)
+    site = tl.site_logliks()
+    np.testing.assert_allclose(site, ora.site_lnl, rtol=10 * LNL_TOL[precision])
+    tl.close()
+
+
+def test_c2_full_size_fp32_and_fp64():
+    """BASELINE configs[2] at full size (1,024-tip Yule, 100,000 patterns)."""
+    w = config_workload("c2", seed=1)
+    ora = oracle_run(w)
+    for precision in (32, 64):
+        tl = gpu_setup(w, "reroot", precision)
+        got = tl.loglik()
+        assert rel(got, ora.lnl) <= LNL_TOL[precision], (precision, got, ora.lnl)
+        tl.close()
+
+
+# ------------------------------------------------------------------ per-node partials
+@pytest.mark.parametrize("precision", [64, 32])
+@pytest.mark.parametrize("kind,n,p", [("pectinate", 128, 2_000), ("yule", 300, 777),
+                                      ("random", 64, 1_001)])
+def test_per_node_partials(precision, kind, n, p):
+    w = make_workload(tree_kind=kind, n=n, p=p, model="gtr", c=4, seed=2, missing_frac=0.05)
+    tl = gpu_setup(w, "reroot", precision)
+    tl.update()
+    ora = oracle_run(w, tree=rooted(tl), keep_partials=True)
+    worst = 0.0
+    for v, L in ora.partials.items():
+        g = tl.partials(v)
+        ge = tl.scale(v - n)                  # cumulative exponents (RRL_FLAG_SCALE_CUMULATIVE)
+        err = node_partial_error(g, ge, L, ora.cum_exponent[v])
+        worst = max(worst, float(err.max()))
+    assert worst <= NODE_TOL[precision], worst
+    tl.close()
+
+
+# ------------------------------------------------------------------ schedules / modes
+def test_schedule_invariance_fp64():
+    w = make_workload(tree_kind="random", n=200, p=3_000, model="gtr", c=4, seed=4)
+    vals = {}
+    for mode in ("sequential", "level", "reroot"):
+        tl = gpu_setup(w, mode, 64)
+        vals[mode] = tl.loglik()
+        tl.close()
+    assert vals["sequential"] == vals["level"]          # same ops, same rooting: bit-identical
+    assert rel(vals["reroot"], vals["level"]) <= 1e-12
+
+
+def test_greedy_batching_and_graph_and_determinism():
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="yule", n=150, p=4_000, model="gtr", c=4, seed=5)
+    tl = gpu_setup(w, "reroot", 32)
+    a = tl.loglik()
+    b = tl.loglik()
+    assert a == b                                        # deterministic
+    R.rrl_update_partials(tl.inst, tl.ops, None)          # greedy sets
+    c = tl.root_loglik()
+    assert c == a
+    tl.close()
+    tg = gpu_setup(w, "reroot", 32, graph=True)
+    assert tg.loglik() == a and tg.loglik() == a         # graph capture, then replay
+    prof = R.rrl_get_profile(tg.inst)
+    assert prof["graph_launches"] == 2
+    tg.close()
+
+
+def test_dependent_ops_in_one_set_rejected():
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="pectinate", n=8, p=64, model="gtr", c=4, seed=1)
+    tl = gpu_setup(w, "level", 32)
+    with pytest.raises(R.RRLError):
+        R.rrl_update_partials(tl.inst, tl.ops, np.array([0, len(tl.ops)], np.int32))
+    tl.close()
+
+
+@pytest.mark.parametrize("precision", [64, 32])
+def test_per_node_scaling_with_accumulate(precision):
+    """Non-cumulative mode: own exponents per node + K5 accumulation."""
+    w = make_workload(tree_kind="random", n=90, p=1_500, model="hky", c=4, seed=7)
+    tl = gpu_setup(w, "reroot", precision, cumulative=False)
+    got = tl.loglik()
+    ora = oracle_run(w, tree=rooted(tl), keep_partials=True)
+    assert rel(got, ora.lnl) <= LNL_TOL[precision]
+    if precision == 64:
+        tot = sum(tl.scale(v - w.n).astype(np.int64) for v in ora.partials)
+        np.testing.assert_array_equal(tot, tl.scale(tl.n_scale - 1))
+    tl.close()
+
+
+def test_buffer_reuse_same_result():
+    w = make_workload(tree_kind="pectinate", n=500, p=2_000, model="gtr", c=4, seed=3)
+    a = gpu_setup(w, "reroot", 32)
+    b = gpu_setup(w, "reroot", 32, reuse=True)
+    assert b.nbuf < a.nbuf
+    la, lb = a.loglik(), b.loglik()
+    assert la == lb
+    a.close()
+    b.close()
+
+
+# ------------------------------------------------------------------ edge cases
+@pytest.mark.parametrize("precision", [64, 32])
+@pytest.mark.parametrize("n,p", [(2, 1), (3, 5), (2, 1000), (5, 129), (17, 257)])
+def test_tiny_and_ragged(precision, n, p):
+    w = make_workload(tree_kind="random", n=n, p=p, model="gtr", c=4, seed=n + p)
+    tl = gpu_setup(w, "reroot", precision)
+    got = tl.loglik()
+    assert rel(got, oracle_run(w).lnl) <= LNL_TOL[precision]
+    tl.close()
+
+
+@pytest.mark.parametrize("c", [1, 2, 8])
+def test_category_counts(c):
+    w = make_workload(tree_kind="yule", n=40, p=500, model="gtr", c=c, seed=c)
+    tl = gpu_setup(w, "reroot", 64)
+    assert rel(tl.loglik(), oracle_run(w).lnl) <= 1e-10
+    tl.close()
+
+
+@pytest.mark.parametrize("precision", [64, 32])
+def test_long_branches_need_scaling(precision):
+    """t = 50 on every branch of a 600-tip tree: lnL_i = sum ln pi_x exactly;
+    the unscaled product underflows fp64, so this exercises the exponents."""
+    w = make_workload(tree_kind="random", n=600, p=300, model="gtr", c=4, seed=8,
+                      missing_frac=0.1)
+    tree = with_blen(w.tree, 50.0)
+    tl = gpu_setup(w, "reroot", precision, tree=tree)
+    got = tl.loglik()
+    pi = w.model.pi
+    exp = math.fsum(math.log(pi[x]) for x in w.tips.ravel() if x < 4)
+    assert rel(got, exp) <= LNL_TOL[precision]
+    tl.close()
+
+
+def test_all_missing_and_zero_branch():
+    w = make_workload(tree_kind="yule", n=30, p=50, model="gtr", c=4, seed=9)
+    w.tips[:, 0] = 4
+    for x in range(4):
+        w.tips[:, 1 + x] = x
+    tl = gpu_setup(w, "reroot", 64)
+    tl.loglik()
+    site = tl.site_logliks()
+    assert abs(site[0]) < 1e-13
+    tl.close()
+    tree = with_blen(w.tree, 0.0)
+    tl = gpu_setup(w, "reroot", 64, tree=tree)
+    tl.loglik()
+    site = tl.site_logliks()
+    for x in range(4):
+        assert abs(site[1 + x] - math.log(w.model.pi[x])) < 1e-13
+    tl.close()
+
+
+def test_tip_partials_equal_tip_states():
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="random", n=20, p=300, model="gtr", c=4, seed=10, missing_frac=0.1)
+    tl = gpu_setup(w, "reroot", 64)
+    a = tl.loglik()
+    for tip in (0, 3, 7):
+        L = pruning.tip_partials(w.tips[tip], 4)
+        R.rrl_set_tip_partials(tl.inst, tip, L)
+    b = tl.loglik()
+    assert rel(b, a) <= 1e-13
+    tl.close()
+
+
+def test_pattern_weights():
+    w = make_workload(tree_kind="random", n=25, p=400, model="gtr", c=4, seed=11)
+    w.pattern_weights = np.random.default_rng(0).integers(1, 5, 400).astype(np.float64)
+    tl = gpu_setup(w, "reroot", 64)
+    assert rel(tl.loglik(), oracle_run(w).lnl) <= 1e-10
+    tl.close()
+
+
+def test_edge_loglik_pulley():
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="balanced", n=32, p=500, model="gtr", c=4, seed=12)
+    tl = gpu_setup(w, "level", 64)
+    root_l = tl.loglik()
+    t = w.tree
+    ch = pruning.children_of(t.parent)
+    a, b = ch[t.root]
+    # matrix for branch a with length t_a + t_b
+    R.rrl_update_transition_matrices(tl.inst, 0, np.array([a], np.int32),
+                                     np.array([t.blen[a] + t.blen[b]]))
+    e = R.rrl_calculate_edge_log_likelihoods(tl.inst, b, a, a, 0, 0, b - w.n, a - w.n)
+    assert rel(e, root_l) <= 1e-12
+    tl.close()

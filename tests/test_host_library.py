@@ -1,0 +1,151 @@
+"""CPU tests of the C-ABI library's host code (no GPU needed).
+
+* every symbol include/rrl.h declares is exported by librrl.so;
+* the C++ O(n) reroot + schedule (rrl_reroot_and_schedule) is bit-exact
+  against the oracle's exhaustive search and its level sets;
+* the C++ model builder + Jacobi eigensystem reproduces the oracle's Q.
+"""
+import ctypes
+import math
+import os
+import re
+
+import numpy as np
+import pytest
+
+from oracle import model as om, reroot as orr
+from workloads import make_tree, random_model
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def R():
+    from paper_conf_ipps_ayresc18_b200 import build
+    build.build()
+    from paper_conf_ipps_ayresc18_b200 import rrl
+    return rrl
+
+
+def test_header_symbols_exported(R):
+    hdr = open(os.path.join(ROOT, "include", "rrl.h")).read()
+    names = set(re.findall(r"\b(rrl_[a-z0-9_]+)\s*\(", hdr))
+    assert len(names) >= 30
+    lib = ctypes.CDLL(R.LIB_PATH)
+    for n in sorted(names):
+        assert hasattr(lib, n), n
+    assert set(R.EXPORTED) == names
+
+
+def test_error_strings(R):
+    assert R.rrl_error_string(R.ERROR_INVALID_TREE) == "invalid tree"
+    assert "sm_100a" in R.rrl_version()
+
+
+def _ops_tuple(ops):
+    return [tuple(int(x) for x in o) for o in ops.tolist()]
+
+
+@pytest.mark.parametrize("kind", ["pectinate", "random", "yule", "balanced"])
+@pytest.mark.parametrize("n", [2, 3, 4, 7, 8, 33, 64, 150])
+def test_reroot_schedule_bit_exact_vs_oracle(R, kind, n):
+    for seed in (1, 2, 3):
+        t = make_tree(kind, n, seed=seed)
+        for mode in ("sequential", "level", "reroot"):
+            rt, ops, offs, key = orr.reroot_and_schedule(t, mode)
+            got = R.rrl_reroot_and_schedule(n, t.parent, t.blen, mode)
+            assert got["root_edge"] == key, (mode, seed)
+            assert np.array_equal(got["parent"], rt.parent)
+            assert np.array_equal(got["blen"], rt.blen)          # bit-exact fp64
+            assert _ops_tuple(got["ops"]) == ops
+            assert got["set_offsets"].tolist() == offs
+            assert got["buffer_count"] == 2 * n - 1
+
+
+@pytest.mark.parametrize("kind", ["random", "yule", "pectinate"])
+def test_edge_table_matches_exhaustive(R, kind):
+    t = make_tree(kind, 120, seed=5)
+    key, sets, imb = R.rrl_reroot_edge_table(120, t.parent)
+    _, _, table = orr.best_rooting(t, with_table=True)
+    exp = sorted((k, s, i) for s, _, i, k in table)
+    assert list(zip(key.tolist(), sets.tolist(), imb.tolist())) == exp
+
+
+def test_large_trees_closed_form(R):
+    """n up to 4096: rerooted set count = ceil((D+1)/2) (survey identity) and
+    the pectinate formulas of PAPER.md:96."""
+    for n in (406, 1024, 4096):
+        t = make_tree("pectinate", n, seed=1)
+        assert R.rrl_reroot_and_schedule(n, t.parent, t.blen, "level")["set_count"] == n - 1
+        g = R.rrl_reroot_and_schedule(n, t.parent, t.blen, "reroot")
+        assert g["set_count"] == math.ceil(n / 2)
+        w = np.diff(g["set_offsets"])
+        assert w.max() == 2 and w.sum() == n - 1
+    for seed in range(1, 6):
+        t = make_tree("random", 1024, seed=seed)
+        g = R.rrl_reroot_and_schedule(1024, t.parent, t.blen, "reroot")
+        assert g["set_count"] == math.ceil((orr.unrooted_diameter(t) + 1) / 2)
+
+
+def test_reuse_buffers_is_a_valid_allocation(R):
+    for kind, n in (("pectinate", 300), ("random", 200), ("yule", 257)):
+        t = make_tree(kind, n, seed=2)
+        full = R.rrl_reroot_and_schedule(n, t.parent, t.blen, "reroot")
+        re_ = R.rrl_reroot_and_schedule(n, t.parent, t.blen, "reroot", reuse_buffers=True)
+        assert re_["buffer_count"] < full["buffer_count"]
+        assert re_["set_offsets"].tolist() == full["set_offsets"].tolist()
+        # simulate: logical node -> physical buffer must hold the value until read
+        phys_of = {}
+        holder = {}
+        offs = re_["set_offsets"]
+        for k in range(len(offs) - 1):
+            lo, hi = offs[k], offs[k + 1]
+            logical = full["ops"][lo:hi]
+            physical = re_["ops"][lo:hi]
+            for lo_op, ph_op in zip(logical, physical):
+                for cl, cp in ((lo_op["child1"], ph_op["child1"]), (lo_op["child2"], ph_op["child2"])):
+                    if cl < n:
+                        assert cp == cl
+                    else:
+                        assert holder[cp] == cl      # still holds the child's value
+                assert ph_op["matrix1"] == lo_op["matrix1"]
+                assert ph_op["dest_scale_write"] == ph_op["dest"] - n
+            dests = set(int(x) for x in physical["dest"])
+            reads = set(int(x) for x in physical["child1"]) | set(int(x) for x in physical["child2"])
+            assert not (dests & reads)
+            for lo_op, ph_op in zip(logical, physical):
+                holder[int(ph_op["dest"])] = int(lo_op["dest"])
+                phys_of[int(lo_op["dest"])] = int(ph_op["dest"])
+        # pectinate rerooted needs only a handful of internal buffers
+        if kind == "pectinate":
+            assert re_["buffer_count"] - n <= 6
+
+
+def test_invalid_trees_rejected(R):
+    t = make_tree("random", 10, seed=1)
+    bad = t.parent.copy()
+    bad[3] = 3
+    with pytest.raises(R.RRLError) as e:
+        R.rrl_reroot_and_schedule(10, bad, t.blen)
+    assert e.value.code == R.ERROR_INVALID_TREE
+    bad = t.parent.copy()
+    bad[bad < 0] = 12          # no root -> cycle
+    with pytest.raises(R.RRLError):
+        R.rrl_reroot_and_schedule(10, bad, t.blen)
+    with pytest.raises(R.RRLError):
+        R.rrl_reroot_and_schedule(1, np.array([-1]), np.array([0.0]))
+
+
+@pytest.mark.parametrize("name", ["jc69", "hky", "gtr", "gy94"])
+def test_model_eigensystem_vs_oracle(R, name):
+    from paper_conf_ipps_ayresc18_b200.engine import model_param_vector
+    mp = random_model(name, np.random.default_rng(17))
+    Q, V, Vi, lam = R.rrl_model_eigensystem(name, mp.pi, model_param_vector(
+        name, mp.kappa, mp.omega, mp.exch))
+    Qo = om.rate_matrix(mp)
+    np.testing.assert_allclose(Q, Qo, atol=1e-14, rtol=1e-12)
+    s = mp.states
+    np.testing.assert_allclose(V @ Vi, np.eye(s), atol=1e-12)
+    np.testing.assert_allclose(V @ np.diag(lam) @ Vi, Qo, atol=1e-12)
+    assert abs(np.sort(lam)[-1]) < 1e-12     # one zero eigenvalue, rest negative
+    assert np.all(np.sort(lam)[:-1] < 0)
