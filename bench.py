@@ -1,0 +1,441 @@
+#!/usr/bin/env python3
+"""Benchmark: rerooted level-batched updatePartials on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config c1] [--precision 32]
+                    [--impl ours|reference]
+
+A "step" is one pass of the whole hot path over the
+workload: K1 transition matrices -> one updatePartials launch per level set
+of the (re)rooted tree (K2; replayed from a CUDA graph) -> root integration K4
+(-> NCCL all-reduce of the fp64 lnL sum when N > 1).  Rerooting + scheduling
+(a1, a2) run once per tree on the host before the timed region, as in the
+paper; the e2e leg repeats them every step.
+
+`value` = effective GFLOPS of Eq. (1) (flops per pattern per pass
+(n-1) c s (4s-1), A16) summed over ranks / max-over-ranks device
+time of the K steps.  Inputs are resident in HBM; L2 (126 MB) is flushed by a
+512 MiB memset before every step, outside the per-step CUDA events.
+
+Multi-GPU: weak scaling -- every rank owns its own 10,000-pattern slice
+(patterns are independent) of a global alignment of N x p
+patterns; the only collective is the all-reduce of the per-rank lnL.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from workloads import CONFIGS, config_workload  # noqa: E402
+
+CONFIG_DESC = {
+    "c0_hky": "configs[0]: 8-tip pectinate, HKY, 1 category, 1,000 patterns",
+    "c1": "configs[1]: 128-tip pectinate rerooted vs original, GTR+G4, 10,000 patterns per GPU",
+    "c2": "configs[2]: 1,024-tip Yule rerooted, GTR+G4, 100,000 patterns per GPU",
+    "c2_paper": "1,024-tip paper-random (PAPER.md:148) rerooted, GTR+G4, 100,000 patterns per GPU",
+    "c4": "configs[4]: 4,096-tip pectinate rerooted, GTR+G4, 4,194,304 patterns (strong scaling)",
+}
+METRIC = "updatePartials GFLOPS rerooted vs original root; %HBM roofline; 1/2/4/8 GPU"
+
+
+def flops_per_pass(n, p, c, s):
+    return (n - 1) * p * c * s * (4 * s - 1)
+
+
+def bytes_per_pass(ops, n, p, c, s, elt, cumulative=True):
+    """Algorithmic HBM bytes of all updatePartials launches of one pass
+    (DESIGN.md §Roofline): per op and pattern, each internal child's c*s*elt
+    partials (+4 B cumulative exponent), each tip child's 1 B state, the
+    c*s*elt output and the 4 B exponent."""
+    per = 0
+    for o in ops:
+        for ch in (int(o["child1"]), int(o["child2"])):
+            per += 1 if ch < n else c * s * elt + (4 if cumulative else 0)
+        per += c * s * elt + 4
+    return per * p
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.rows = []
+        self.proc = None
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-i", str(device), "-lms", "100"], stdout=subprocess.PIPE,
+                stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append(line.strip())
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            parts = [x.strip() for x in r.split(",")]
+            if len(parts) != 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[2:]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None,
+                "sm_max_mhz": float(max(mx)) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------------- helpers
+def rank_workload(cfg: str, rank: int, world: int, seed: int = 1):
+    """Weak scaling (c0-c2): each rank owns patterns [r p, (r+1) p) of a global
+    alignment of world*p patterns.  Strong scaling (c4): the global p is split."""
+    base = dict(CONFIGS[cfg])
+    p = base["p"]
+    if cfg == "c4":
+        chunk = math.ceil(p / world)
+        lo, hi = rank * chunk, min(p, (rank + 1) * chunk)
+        w = config_workload(cfg, seed=seed, p=1)           # tree + model only
+        rng = np.random.default_rng(np.random.SeedSequence([seed, 7919, rank]))
+        w.tips = rng.integers(0, w.s, size=(w.n, hi - lo), dtype=np.uint8)
+        w.pattern_weights = np.ones(hi - lo)
+        return w, "strong"
+    w = config_workload(cfg, seed=seed, p=p * world)
+    w.tips = np.ascontiguousarray(w.tips[:, rank * p:(rank + 1) * p])
+    w.pattern_weights = np.ones(p)
+    return w, "weak"
+
+
+def ncu_traffic(cfg: str, precision: int):
+    """DRAM bytes per updatePartials launch from the committed ncu capture."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        d = json.load(open(path))
+        return d.get(f"{cfg}_fp{precision}")
+    except Exception:
+        return None
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "measured"
+    except Exception:
+        return {"hbm_gbs": 6650.0}, "fallback"
+
+
+# ----------------------------------------------------------------------------- reference arm
+def run_reference(args, rank, world):
+    """--impl reference: the fp64 oracle (test infrastructure) timed as it
+    stands on the host cores, on a bounded pattern sample of the workload."""
+    if rank != 0:
+        return
+    from threadpoolctl import threadpool_limits
+
+    from oracle import model as om, pruning
+    w, _ = rank_workload(args.config, 0, 1)
+    sample = min(w.p, args.ref_patterns)
+    tips = np.ascontiguousarray(w.tips[:, :sample])
+    pw = np.ones(sample)
+    Q = om.rate_matrix(w.model)
+    fl = flops_per_pass(w.n, sample, w.c, w.s)
+    with threadpool_limits(limits=1):
+        t0 = time.perf_counter()
+        pruning.prune(w.tree, Q, w.model.pi, w.rates, w.cat_weights, tips, pw)
+        est = (time.perf_counter() - t0) * (args.steps + args.warmup)
+        if est > 150.0:  # keep the whole reference run within a few minutes
+            sample = max(256, int(sample * 150.0 / est))
+            tips = np.ascontiguousarray(w.tips[:, :sample])
+            pw = np.ones(sample)
+            fl = flops_per_pass(w.n, sample, w.c, w.s)
+        for _ in range(args.warmup):
+            pruning.prune(w.tree, Q, w.model.pi, w.rates, w.cat_weights, tips, pw)
+        t0 = time.perf_counter()
+        for _ in range(args.steps):
+            pruning.prune(w.tree, Q, w.model.pi, w.rates, w.cat_weights, tips, pw)
+        dt = time.perf_counter() - t0
+    val = fl * args.steps / dt / 1e9
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": "GFLOPS",
+        "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+        "ms_per_step": dt / args.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded, workloads/)",
+        "config": {"workload": CONFIG_DESC.get(args.config, args.config),
+                   "sample_patterns": sample, "schedule": "post-order (oracle)"},
+        "cpu_baseline": {"value": val, "unit": "GFLOPS", "cores": 1, "kind": "oracle",
+                         "sample": f"{sample} of {w.p} patterns, full {w.n}-tip tree, per step"},
+        "e2e": {"value": val, "unit": "GFLOPS", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def cpu_baseline(w, budget_s=15.0):
+    """The oracle as it stands on one host core, on a bounded pattern sample."""
+    from threadpoolctl import threadpool_limits
+
+    from oracle import model as om, pruning
+    Q = om.rate_matrix(w.model)
+    sample = min(w.p, 2000)
+    tips = np.ascontiguousarray(w.tips[:, :sample])
+    pw = np.ones(sample)
+    reps, t_total = 0, 0.0
+    with threadpool_limits(limits=1):
+        while t_total < budget_s and reps < 50:
+            t0 = time.perf_counter()
+            pruning.prune(w.tree, Q, w.model.pi, w.rates, w.cat_weights, tips, pw)
+            t_total += time.perf_counter() - t0
+            reps += 1
+    val = flops_per_pass(w.n, sample, w.c, w.s) * reps / t_total / 1e9
+    return {"value": val, "unit": "GFLOPS", "cores": 1, "kind": "oracle",
+            "sample": f"{reps} passes x {sample} of {w.p} patterns, full {w.n}-tip tree "
+                      f"({t_total:.1f} s, numpy/scipy fp64, 1 thread)"}
+
+
+# ----------------------------------------------------------------------------- our arm
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--warmup", type=int, default=10)
+    ap.add_argument("--config", default="c1", choices=sorted(CONFIG_DESC))
+    ap.add_argument("--precision", type=int, default=32, choices=(32, 64))
+    ap.add_argument("--impl", default="ours", choices=("ours", "reference"))
+    ap.add_argument("--no-graph", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--ref-patterns", type=int, default=10_000)
+    args = ap.parse_args()
+    args.warmup = max(args.warmup, 3)
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+
+    import torch
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
+    torch.cuda.set_device(local)
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    from paper_conf_ipps_ayresc18_b200 import build as _b
+    _b.build()
+    from paper_conf_ipps_ayresc18_b200 import TreeLikelihood, rrl as R
+
+    w, scaling = rank_workload(args.config, rank, world)
+    n, p, c, s = w.n, w.p, w.c, w.s
+    elt = 4 if args.precision == 32 else 8
+    stream = torch.cuda.current_stream()
+    reuse = args.config == "c4"
+
+    def make(mode):
+        nbuf = None
+        if reuse:
+            nbuf = R.rrl_reroot_and_schedule(n, w.tree.parent, w.tree.blen, mode, True)["buffer_count"]
+        tl = TreeLikelihood(n, p, s, c, precision=args.precision, device=local,
+                            cuda_graph=not args.no_graph, buffer_count=nbuf,
+                            stream_ptr=stream.cuda_stream)
+        tl.set_model_params(w.model, w.rates, w.cat_weights)
+        tl.set_tips(w.tips)
+        tl.set_pattern_weights(w.pattern_weights)
+        tl.set_tree(w.tree.parent, w.tree.blen, mode, reuse_buffers=reuse)
+        return tl
+
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    d_out = torch.zeros(1, dtype=torch.float64, device="cuda")
+
+    def step(tl):
+        tl.update()
+        tl.root_loglik_device(d_out.data_ptr())
+        if dist is not None:
+            dist.all_reduce(d_out)
+
+    def timed(tl, steps, warmup):
+        for _ in range(warmup):
+            flush.zero_()
+            step(tl)
+        torch.cuda.synchronize()
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in range(steps)]
+        R.rrl_reset_profile(tl.inst)
+        for a, b in evs:
+            flush.zero_()
+            a.record(stream)
+            step(tl)
+            b.record(stream)
+        torch.cuda.synchronize()
+        if dist is not None:
+            dist.barrier()
+        torch.cuda.synchronize()
+        ms = sum(a.elapsed_time(b) for a, b in evs)
+        launches = R.rrl_get_profile(tl.inst)["kernel_launches"]
+        return ms, launches
+
+    def maxall(x):
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def instrumented(tl, steps):
+        """Per-launch CUDA events (library profiling mode, eager launches) on
+        the launching stream: durations of every updatePartials launch."""
+        R.rrl_set_profiling(tl.inst, True)
+        R.rrl_reset_profile(tl.inst)
+        for _ in range(steps):
+            flush.zero_()
+            step(tl)
+        prof = R.rrl_get_profile(tl.inst)
+        R.rrl_set_profiling(tl.inst, False)
+        return prof
+
+    # ---- rerooted (the product configuration)
+    tl = make("reroot")
+    sched = tl.sched
+    clocks = ClockSampler(local)
+    ms, launches = timed(tl, args.steps, args.warmup)
+    clk = clocks.stop()
+    ms_max = maxall(ms)
+    fl = flops_per_pass(n, p, c, s)
+    value = fl * world * args.steps / (ms_max * 1e-3) / 1e9
+    prof = instrumented(tl, min(args.steps, 100))
+    nsteps_i = min(args.steps, 100)
+    part_ms = prof["partials_ms"] / nsteps_i
+    nlaunch = prof["partials_launches"] / nsteps_i
+    bpp = bytes_per_pass(sched["ops"], n, p, c, s, elt)
+    achieved = bpp / (part_ms * 1e-3) / 1e9
+    peaks, peak_src = measured_peaks()
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
+    traffic = ncu_traffic(args.config, args.precision)
+    lnl = float(d_out.item())
+
+    # ---- original rooting, same kernels (the reroot speedup of the paper)
+    orig = {}
+    if args.config != "c4":
+        to = make("level")
+        ms_o, _ = timed(to, args.steps, args.warmup)
+        ms_o = maxall(ms_o)
+        prof_o = instrumented(to, nsteps_i)
+        orig = {"sets": to.sched["set_count"], "gflops": fl * world * args.steps / (ms_o * 1e-3) / 1e9,
+                "ms_per_step": ms_o / args.steps,
+                "updatePartials_ms": prof_o["partials_ms"] / nsteps_i}
+        to.close()
+
+    # ---- e2e through the public API with host buffers (pinned), every step:
+    # reroot + schedule, H2D tips + branch lengths, pass, D2H of the lnL.
+    pinned = torch.empty(w.tips.shape, dtype=torch.uint8, pin_memory=True).numpy()
+    pinned[:] = w.tips
+    e2e_steps = max(3, min(args.steps, 50))
+    for _ in range(2):
+        tl.set_tips(pinned)
+        tl.set_tree(w.tree.parent, w.tree.blen, "reroot", reuse_buffers=reuse)
+        tl.loglik()
+    torch.cuda.synchronize()
+    if dist is not None:
+        dist.barrier()
+    t0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        tl.set_tips(pinned)
+        tl.set_tree(w.tree.parent, w.tree.blen, "reroot", reuse_buffers=reuse)
+        tl.update()
+        tl.root_loglik_device(d_out.data_ptr())
+        if dist is not None:
+            dist.all_reduce(d_out)
+        host_l = float(d_out.item())
+    e2e_s = maxall(time.perf_counter() - t0)
+    e2e_val = fl * world * e2e_steps / e2e_s / 1e9
+    h2d = int(w.tips.nbytes + tl.t.nbytes + tl.matrix_idx.nbytes)
+    tl.close()
+
+    if rank != 0:
+        return
+    cpu = None if args.no_cpu_baseline else cpu_baseline(w)
+    out = {
+        "metric": METRIC,
+        "value": value,
+        "unit": "GFLOPS",
+        "n_gpus": world,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": ms_max / args.steps,
+        "higher_is_better": True,
+        "scaling": scaling,
+        "vs_baseline": None,
+        "dtype": f"f{args.precision}",
+        "data": "synthetic (seeded workloads/: tree, GTR+G4 parameters, uniform alignment)",
+        "config": {"workload": CONFIG_DESC[args.config], "n_tips": n, "patterns_per_gpu": p,
+                   "categories": c, "states": s, "schedule": "reroot", "sets": sched["set_count"],
+                   "cuda_graph": not args.no_graph,
+                   "l2": "flushed before every step (512 MiB memset, outside the step events)"},
+        "reroot": {"sets": sched["set_count"], "sets_original": orig.get("sets"),
+                   "theoretical_speedup": (orig["sets"] / sched["set_count"]) if orig else None,
+                   "step_speedup": (ms_o / ms_max) if orig else None,
+                   "updatePartials_speedup": (orig["updatePartials_ms"] / part_ms) if orig else None,
+                   "original_gflops": orig.get("gflops"),
+                   "paper_context": "BEAGLE CUDA on Quadro GP100: up to 1.93x (pectinate, 406 OTUs, "
+                                    "512 patterns, PAPER.md:258); mean 1.26x (random 256 OTUs, PAPER.md:230)"},
+        "updatePartials": {"ms_per_pass": part_ms, "launches_per_pass": nlaunch,
+                           "gflops": fl / (part_ms * 1e-3) / 1e9,
+                           "pattern_node_updates_per_s": (n - 1) * p / (part_ms * 1e-3),
+                           "share_of_step": part_ms / (ms_max / args.steps)},
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                     "frac": achieved / hbm, "traffic": traffic,
+                     "kernel": "k_partials_nuc (updatePartials, one launch per level set)",
+                     "algorithmic_bytes_per_pass": bpp,
+                     "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json)",
+                     "timing": "per-launch CUDA events on the launching stream, eager "
+                               f"instrumented pass of {nsteps_i} steps after the timed region"},
+        "cpu_baseline": cpu,
+        "e2e": {"value": e2e_val, "unit": "GFLOPS", "h2d_bytes_per_step": h2d,
+                "d2h_bytes_per_step": 8, "steps": e2e_steps,
+                "path": "TreeLikelihood: set_tips (pinned H2D) + rrl_reroot_and_schedule + K1 + "
+                        "level-set K2 + K4 + D2H lnL"},
+        "gpu_launches": int(launches),
+        "clocks": clk,
+        "lnL": lnl,
+    }
+    print(json.dumps(out), flush=True)
+    if dist is not None:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

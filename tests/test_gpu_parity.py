@@ -187,9 +187,9 @@ def test_category_counts(c):
 def test_long_branches_need_scaling(precision):
     """t = 50 on every branch of a 600-tip tree: lnL_i = sum ln pi_x exactly;
     the unscaled product underflows fp64, so this exercises the exponents."""
-    w = make_workload(tree_kind="random", n=600, p=300, model="gtr", c=4, seed=8,
+    w = make_workload(tree_kind="random", n=600, p=300, model="gtr", c=1, seed=8,
                       missing_frac=0.1)
-    tree = with_blen(w.tree, 50.0)
+    tree = with_blen(w.tree, 50.0)  # c = 1: rate 1, so every P is at its t -> inf limit
     tl = gpu_setup(w, "reroot", precision, tree=tree)
     got = tl.loglik()
     pi = w.model.pi
