@@ -139,8 +139,11 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
                         int precision, uint32_t flags);
 int rrl_finalize_instance(int inst);
 
-/* Use the caller's CUDA stream (e.g. torch.cuda.current_stream().cuda_stream);
- * NULL restores the instance's own stream. */
+/* Enqueue all later work on the caller's CUDA stream (e.g.
+ * torch.cuda.current_stream().cuda_stream).  The stream is used as given:
+ * NULL is the legacy default stream (RRL_FLAG_CUDA_GRAPH then launches
+ * eagerly, since the legacy stream cannot be captured).  Until this is
+ * called the instance uses its own non-blocking stream. */
 int rrl_set_stream(int inst, void *cuda_stream);
 int rrl_synchronize(int inst);
 

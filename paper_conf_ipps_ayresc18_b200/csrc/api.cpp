@@ -57,6 +57,7 @@ struct Instance {
   double *d_site = nullptr;              // [p_pad]
   double *d_block = nullptr;             // [nblocks]
   double *d_out = nullptr;               // scalar
+  unsigned *d_count = nullptr;           // last-block-done ticket of K4/K6
   double *h_out = nullptr;               // pinned scalar
   int nblocks = 0;
 
@@ -180,7 +181,7 @@ void destroy(Instance *I) {
   for (void *t : I->tip_partials)
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
-                  I->d_catw,     I->d_freqs,  I->d_pw,   I->d_site,  I->d_block, I->d_out,
+                  I->d_catw,     I->d_freqs,  I->d_pw,   I->d_site,  I->d_block, I->d_out, I->d_count,
                   I->d_midx,     I->d_t,      I->d_sidx, I->d_ops};
   for (void *q : ptrs)
     if (q) cudaFree(q);
@@ -332,6 +333,8 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
   CKC(cudaMalloc(&I->d_site, sizeof(double) * I->p_pad));
   CKC(cudaMalloc(&I->d_block, sizeof(double) * I->nblocks));
   CKC(cudaMalloc(&I->d_out, sizeof(double)));
+  CKC(cudaMalloc(&I->d_count, sizeof(unsigned)));
+  CKC(cudaMemset(I->d_count, 0, sizeof(unsigned)));
   CKC(cudaMallocHost(&I->h_out, sizeof(double)));
   {
     std::vector<double> ones(I->p_pad, 1.0), r(category_count, 1.0),
@@ -363,7 +366,7 @@ int rrl_finalize_instance(int inst) {
 
 int rrl_set_stream(int inst, void *cuda_stream) {
   GET(I, inst);
-  cudaStream_t ns = cuda_stream ? static_cast<cudaStream_t>(cuda_stream) : I->own_stream;
+  cudaStream_t ns = static_cast<cudaStream_t>(cuda_stream);  // NULL = legacy default stream
   if (ns != I->stream) {
     CK(cudaStreamSynchronize(I->stream));
     I->stream = ns;
@@ -686,10 +689,10 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
     for (int k = 0; k < nsets; ++k) {
       const int n = offs[k + 1] - offs[k];
       Timed tm(I, 0);
-      int e = (I->s == 4) ? launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k], n, I->p,
-                                                       I->p_pad, I->stream)
-                          : launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k], n, I->p,
-                                                         I->p_pad, I->stream);
+      int e = (I->s == 4) ? launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k],
+                                                       I->h_ops + offs[k], n, I->p, I->p_pad, I->stream)
+                          : launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k],
+                                                         I->h_ops + offs[k], n, I->p, I->p_pad, I->stream);
       if (e == (int)cudaErrorNotSupported) return fail(RRL_ERROR_NO_IMPLEMENTATION, "kernel variant");
       if (e != 0) return fail(RRL_ERROR_CUDA, std::string("updatePartials launch: ") +
                                                   cudaGetErrorString(static_cast<cudaError_t>(e)));
@@ -697,7 +700,8 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
     return 0;
   };
 
-  const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && !I->profiling;
+  // (the legacy default stream cannot be captured: eager launches there)
+  const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && !I->profiling && I->stream != nullptr;
   if (use_graph) {
     if (I->graph && I->graph_stream != I->stream) {
       cudaGraphExecDestroy(I->graph);
@@ -791,10 +795,10 @@ static int root_common(Instance *I, int root_buffer, int cat_weights_idx, int fr
     Timed tm(I, 2);
     CKL(launch_root_lnl(I->prec, I->s, I->s_pad, I->c, root, I->d_catw + (size_t)cat_weights_idx * I->c,
                         I->d_freqs + (size_t)freqs_idx * I->s, cum, I->d_pw, I->p, I->p_pad, I->d_site,
-                        I->d_block, I->nblocks, d_out, I->stream));
+                        I->d_block, I->d_count, I->nblocks, d_out, I->stream));
   }
-  I->prof.root_launches += 2;
-  I->prof.kernel_launches += 2;
+  I->prof.root_launches += 1;
+  I->prof.kernel_launches += 1;
   return RRL_SUCCESS;
 }
 
@@ -844,11 +848,11 @@ int rrl_calculate_edge_log_likelihoods(int inst, int parent_buffer, int child_bu
     CKL(launch_edge_lnl(I->prec, I->s, I->s_pad, I->c, par, child, tip ? 1 : 0,
                         I->d_P + (size_t)matrix_idx * I->mat_elems * I->elt,
                         I->d_catw + (size_t)cat_weights_idx * I->c, I->d_freqs + (size_t)freqs_idx * I->s,
-                        cp, cc, I->d_pw, I->p, I->p_pad, I->d_site, I->d_block, I->nblocks, I->d_out,
+                        cp, cc, I->d_pw, I->p, I->p_pad, I->d_site, I->d_block, I->d_count, I->nblocks, I->d_out,
                         I->stream));
   }
-  I->prof.root_launches += 2;
-  I->prof.kernel_launches += 2;
+  I->prof.root_launches += 1;
+  I->prof.kernel_launches += 1;
   CK(cudaMemcpyAsync(I->h_out, I->d_out, sizeof(double), cudaMemcpyDeviceToHost, I->stream));
   CK(cudaStreamSynchronize(I->stream));
   *out_sum = *I->h_out;

@@ -6,7 +6,7 @@
 
 namespace rrl {
 
-int launch_update_partials_codon(int, int, const DevOp *, int, int, int, void *) {
+int launch_update_partials_codon(int, int, const DevOp *, const DevOp *, int, int, int, void *) {
   return (int)cudaErrorNotSupported;
 }
 

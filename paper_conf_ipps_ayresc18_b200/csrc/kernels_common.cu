@@ -67,6 +67,30 @@ __device__ double block_sum(double v, double *red) {
   return r;  // valid in thread 0
 }
 
+// Each block publishes its partial sum; the last block to finish (ticket)
+// adds all of them in block order, so the result is deterministic for a
+// fixed grid, with a single launch (no separate final-reduction kernel).
+__device__ void finish_sum(double part, double *red, double *blocks, unsigned *count, double *out) {
+  __shared__ bool last;
+  const double r = block_sum(part, red);
+  if (threadIdx.x == 0) {
+    blocks[blockIdx.x] = r;
+    __threadfence();
+    last = atomicAdd(count, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!last) return;
+  __threadfence();
+  double v = 0.0;
+  for (int i = threadIdx.x; i < (int)gridDim.x; i += blockDim.x) v += ((volatile double *)blocks)[i];
+  __syncthreads();
+  const double tot = block_sum(v, red);
+  if (threadIdx.x == 0) {
+    *out = tot;
+    *count = 0u;
+  }
+}
+
 template <typename T>
 __device__ inline double site_root(const T *L, int s, int s_pad, int C, int i, int p_pad,
                                    const double *w, const double *pi) {
@@ -88,7 +112,7 @@ __global__ void __launch_bounds__(256)
 k_root(const T *__restrict__ L, int s, int s_pad, int C, const double *__restrict__ w,
        const double *__restrict__ pi, const int32_t *__restrict__ cum,
        const double *__restrict__ pw, int p, int p_pad, double *__restrict__ site,
-       double *__restrict__ blocks) {
+       double *__restrict__ blocks, unsigned *__restrict__ count, double *__restrict__ out) {
   __shared__ double red[32];
   double part = 0.0;
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < p; i += gridDim.x * blockDim.x) {
@@ -98,16 +122,7 @@ k_root(const T *__restrict__ L, int s, int s_pad, int C, const double *__restric
     site[i] = l;
     part += pw[i] * l;
   }
-  const double r = block_sum(part, red);
-  if (threadIdx.x == 0) blocks[blockIdx.x] = r;
-}
-
-__global__ void k_final(const double *__restrict__ blocks, int nb, double *__restrict__ out) {
-  __shared__ double red[32];
-  double v = 0.0;
-  for (int i = threadIdx.x; i < nb; i += blockDim.x) v += blocks[i];
-  const double r = block_sum(v, red);
-  if (threadIdx.x == 0) *out = r;
+  finish_sum(part, red, blocks, count, out);
 }
 
 // ---------------------------------------------------------------------- K6
@@ -117,7 +132,8 @@ k_edge(const T *__restrict__ Lp, const void *__restrict__ child, int child_is_ti
        const T *__restrict__ P, int s, int s_pad, int C, const double *__restrict__ w,
        const double *__restrict__ pi, const int32_t *__restrict__ cum_p,
        const int32_t *__restrict__ cum_c, const double *__restrict__ pw, int p, int p_pad,
-       double *__restrict__ site, double *__restrict__ blocks) {
+       double *__restrict__ site, double *__restrict__ blocks, unsigned *__restrict__ count,
+       double *__restrict__ out) {
   __shared__ double red[32];
   double part = 0.0;
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < p; i += gridDim.x * blockDim.x) {
@@ -150,8 +166,7 @@ k_edge(const T *__restrict__ Lp, const void *__restrict__ child, int child_is_ti
     site[i] = l;
     part += pw[i] * l;
   }
-  const double r = block_sum(part, red);
-  if (threadIdx.x == 0) blocks[blockIdx.x] = r;
+  finish_sum(part, red, blocks, count, out);
 }
 
 }  // namespace
@@ -191,32 +206,32 @@ int launch_accumulate_scale(const int32_t *d_scale, int p_pad, const int32_t *d_
 
 int launch_root_lnl(int prec, int s, int s_pad, int c, const void *root, const double *d_w,
                     const double *d_pi, const int32_t *cum, const double *d_pw, int p, int p_pad,
-                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream) {
+                    double *d_site, double *d_block, unsigned *d_count, int nblocks, double *d_out,
+                    void *stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (prec == 32)
     k_root<float><<<nblocks, 256, 0, st>>>(static_cast<const float *>(root), s, s_pad, c, d_w, d_pi,
-                                           cum, d_pw, p, p_pad, d_site, d_block);
+                                           cum, d_pw, p, p_pad, d_site, d_block, d_count, d_out);
   else
     k_root<double><<<nblocks, 256, 0, st>>>(static_cast<const double *>(root), s, s_pad, c, d_w, d_pi,
-                                            cum, d_pw, p, p_pad, d_site, d_block);
-  k_final<<<1, 256, 0, st>>>(d_block, nblocks, d_out);
+                                            cum, d_pw, p, p_pad, d_site, d_block, d_count, d_out);
   return (int)cudaGetLastError();
 }
 
 int launch_edge_lnl(int prec, int s, int s_pad, int c, const void *par, const void *child,
                     int child_is_tip, const void *P, const double *d_w, const double *d_pi,
                     const int32_t *cum_p, const int32_t *cum_c, const double *d_pw, int p, int p_pad,
-                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream) {
+                    double *d_site, double *d_block, unsigned *d_count, int nblocks, double *d_out,
+                    void *stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (prec == 32)
     k_edge<float><<<nblocks, 256, 0, st>>>(static_cast<const float *>(par), child, child_is_tip,
                                            static_cast<const float *>(P), s, s_pad, c, d_w, d_pi,
-                                           cum_p, cum_c, d_pw, p, p_pad, d_site, d_block);
+                                           cum_p, cum_c, d_pw, p, p_pad, d_site, d_block, d_count, d_out);
   else
     k_edge<double><<<nblocks, 256, 0, st>>>(static_cast<const double *>(par), child, child_is_tip,
                                             static_cast<const double *>(P), s, s_pad, c, d_w, d_pi,
-                                            cum_p, cum_c, d_pw, p, p_pad, d_site, d_block);
-  k_final<<<1, 256, 0, st>>>(d_block, nblocks, d_out);
+                                            cum_p, cum_c, d_pw, p, p_pad, d_site, d_block, d_count, d_out);
   return (int)cudaGetLastError();
 }
 

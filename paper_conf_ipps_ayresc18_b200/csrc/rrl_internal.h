@@ -34,10 +34,12 @@ enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2 };
 
 // ---------------------------------------------------------------- launchers
 // All launchers enqueue on `stream` and return cudaError_t as int.
-int launch_update_partials_nuc(int prec, int c, const DevOp *ops, int nops, int p, int p_pad,
-                               void *stream);
-int launch_update_partials_codon(int prec, int c, const DevOp *ops, int nops, int p, int p_pad,
-                                 void *stream);
+// d_ops: descriptors in device memory; h_ops: the same descriptors on the host
+// (small sets are passed by value in the kernel parameters), may be null.
+int launch_update_partials_nuc(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
+                               int p, int p_pad, void *stream);
+int launch_update_partials_codon(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
+                                 int p, int p_pad, void *stream);
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
                                int count, void *d_P, void *stream);
@@ -45,10 +47,12 @@ int launch_accumulate_scale(const int32_t *d_scale, int p_pad, const int32_t *d_
                             int32_t *d_cum, int p, void *stream);
 int launch_root_lnl(int prec, int s, int s_pad, int c, const void *root, const double *d_w,
                     const double *d_pi, const int32_t *cum, const double *d_pw, int p, int p_pad,
-                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream);
+                    double *d_site, double *d_block, unsigned *d_count, int nblocks, double *d_out,
+                    void *stream);
 int launch_edge_lnl(int prec, int s, int s_pad, int c, const void *par, const void *child,
                     int child_is_tip, const void *P, const double *d_w, const double *d_pi,
                     const int32_t *cum_p, const int32_t *cum_c, const double *d_pw, int p, int p_pad,
-                    double *d_site, double *d_block, int nblocks, double *d_out, void *stream);
+                    double *d_site, double *d_block, unsigned *d_count, int nblocks, double *d_out,
+                    void *stream);
 
 }  // namespace rrl

@@ -203,14 +203,18 @@ def test_all_missing_and_zero_branch():
     w.tips[:, 0] = 4
     for x in range(4):
         w.tips[:, 1 + x] = x
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
     tl = gpu_setup(w, "reroot", 64)
     tl.loglik()
     site = tl.site_logliks()
     assert abs(site[0]) < 1e-13
     tl.close()
-    tree = with_blen(w.tree, 0.0)
+    tree = with_blen(w.tree, 0.0)          # non-constant patterns get L = 0 -> lnL = -inf
     tl = gpu_setup(w, "reroot", 64, tree=tree)
-    tl.loglik()
+    tl.update()
+    total = R.rrl_calculate_root_log_likelihoods(tl.inst, tl.root_buffer, 0, 0, tl.cumulative_idx,
+                                                 allow_nonfinite=True)
+    assert np.isneginf(total)
     site = tl.site_logliks()
     for x in range(4):
         assert abs(site[1 + x] - math.log(w.model.pi[x])) < 1e-13
