@@ -287,7 +287,7 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
   I->s = state_count;
   I->s_pad = state_count == 4 ? 4 : 64;
   I->p = pattern_count;
-  I->p_pad = (pattern_count + 127) / 128 * 128;
+  I->p_pad = (pattern_count + 511) / 512 * 512;  // whole bulk-copy chunks (kernels_nuc.cu)
   I->c = category_count;
   I->n_mat = matrix_count;
   I->n_eig = eigen_count;

@@ -1,30 +1,34 @@
 // K2: level-set updatePartials for 4-state models (sm_100a).
 //
 // Eq. (1) (§II-A) for every operation of one concurrent set in a
-// single launch (§VI-A multi-operation kernel): grid.y indexes
-// the operation, grid.x strides over pattern chunks.  Device layout [p][c][4]:
-// one thread owns one (pattern, category) pair, i.e. one 16-byte (fp32) or
-// 32-byte (fp64) state vector per child, so a warp moves 512 contiguous bytes
-// per child per item with 128-bit loads; U items per thread are loaded before
-// any is consumed.  The two 4x4 transition matrices of the thread's category
-// live in registers (loaded once per block); tip children are uint8 state
-// codes resolved by selecting a column of P (code 4 = missing -> the row sum,
-// i.e. an all-ones partial vector).
+// single launch (§VI-A multi-operation kernel).  Device layout
+// [p][c][4]: one thread owns one (pattern, category) item, i.e. one 16-byte
+// (fp32) or 32-byte (fp64) state vector per child.  The two 4x4 transition
+// matrices of an operation sit in shared memory twice: row-major for the
+// internal-child mat-vec and column-major (plus the row-sum column) so that a
+// tip child's contribution P[.][state] is a single 128-bit LDS (state code 4 =
+// missing -> the row sums, i.e. an all-ones partial vector).
 //
 // Rescaling (reading A5) is fused: the C lanes of a pattern
 // reduce max over (c, z) with warp shuffles, the frexp exponent e is read from
 // the float's exponent bits, the outputs are multiplied by 2^-e (exact) and e
 // (own, or own + children's cumulative) is stored as int32.
 //
-// Launch-latency path (narrow sets, e.g. 2 ops per set for a rerooted
-// pectinate tree): operation descriptors for sets of <= kInline ops travel in
-// the kernel parameters (no dependent descriptor load), and launches use
-// programmatic dependent launch: a block resolves its descriptor, then waits
-// (griddepcontrol.wait) for the previous level set before touching P or any
-// partials, then lets the next set's grid start launching.
+// Two variants, chosen per launch by the host:
+//  * k_partials_nuc (latency path, narrow sets / few patterns): grid
+//    (pattern chunks x ops); descriptors of sets of <= kInline ops travel in
+//    the kernel parameters; child vectors are loaded straight into registers.
+//  * k_partials_nuc_bulk (bandwidth path, many patterns): persistent blocks
+//    walk a contiguous range of the flattened (op, chunk) space; one thread
+//    streams each chunk's child partials / tip states / child exponents into
+//    a kStages-deep shared-memory ring with cp.async.bulk (TMA bulk copies,
+//    mbarrier completion) while all threads compute the previous stage, so
+//    bytes in flight no longer depend on registers per thread.
+// Both use programmatic dependent launch: the prologue overlaps the previous
+// level set; griddepcontrol.wait precedes every read of P or partials.
 //
-// HBM-bound for wide sets: per (pattern, op) 2 x c x 4 x sizeof(T) child bytes
-// (tips: 1 B) + c x 4 x sizeof(T) out + exponents; 1.8 flop/B in fp32.
+// HBM-bound: per (pattern, op) 2 x c x 4 x sizeof(T) child bytes (tips: 1 B)
+// + c x 4 x sizeof(T) out + exponents; 1.8 flop/B in fp32.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -36,6 +40,8 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kInline = 8;
+constexpr int kChunkItems = 512;  // items (pattern x category) per bulk chunk
+constexpr int kPTab = 36;         // per (branch, cat): 16 rows P[z][x] + 5 columns x 4
 
 struct OpPack {
   const DevOp *ops;  // used when n > kInline
@@ -49,12 +55,12 @@ template <> struct V4<float> {
     const float4 x = __ldg(reinterpret_cast<const float4 *>(p));
     v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
   }
-  __device__ static inline void st(float *p, const float (&v)[4]) {
-    *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
-  }
   __device__ static inline void lds(const float *p, float (&v)[4]) {
     const float4 x = *reinterpret_cast<const float4 *>(p);
     v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+  }
+  __device__ static inline void st(float *p, const float (&v)[4]) {
+    *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]);
   }
 };
 template <> struct V4<double> {
@@ -63,19 +69,18 @@ template <> struct V4<double> {
     const double2 b = __ldg(reinterpret_cast<const double2 *>(p) + 1);
     v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
   }
-  __device__ static inline void st(double *p, const double (&v)[4]) {
-    reinterpret_cast<double2 *>(p)[0] = make_double2(v[0], v[1]);
-    reinterpret_cast<double2 *>(p)[1] = make_double2(v[2], v[3]);
-  }
   __device__ static inline void lds(const double *p, double (&v)[4]) {
     const double2 a = reinterpret_cast<const double2 *>(p)[0];
     const double2 b = reinterpret_cast<const double2 *>(p)[1];
     v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
   }
+  __device__ static inline void st(double *p, const double (&v)[4]) {
+    reinterpret_cast<double2 *>(p)[0] = make_double2(v[0], v[1]);
+    reinterpret_cast<double2 *>(p)[1] = make_double2(v[2], v[3]);
+  }
 };
 
-// frexp exponent e (m = f 2^e, f in [0.5,1)) and the exact factor 2^-e.
-// Fast path from the exponent bits for normal m; library fallback otherwise.
+// frexp exponent e (m = f 2^e, f in [0.5,1)), fast path from the exponent bits.
 __device__ inline int frexp_exp(float m) {
   const unsigned b = __float_as_uint(m);
   const int eb = (int)((b >> 23) & 0xffu);
@@ -94,6 +99,7 @@ __device__ inline int frexp_exp(double m) {
   frexp(m, &e);
   return e;
 }
+// r *= 2^-e, exactly.
 __device__ inline void scale_pow2(float (&r)[4], int e) {
   if (e > -126 && e < 126) {
     const float f = __uint_as_float((unsigned)(127 - e) << 23);
@@ -115,15 +121,27 @@ __device__ inline void scale_pow2(double (&r)[4], int e) {
   }
 }
 
-// P rows of one (branch, category) in shared memory: 16 entries P[z][x] then
-// the 4 row sums (the tip lookup of a missing state).  Stride 20 keeps the
-// LDS.128 rows of the C categories a warp touches in distinct banks.
-constexpr int kPStride = 20;
+// Shared-memory transition tables of one operation: [branch][cat][kPTab].
+template <typename T, int C>
+__device__ inline void load_ptables(T (*sP)[C][kPTab], const DevOp &op) {
+  for (int t = threadIdx.x; t < 2 * C * 16; t += blockDim.x) {
+    const int b = t / (C * 16), r = t % (C * 16), c = r / 16, zx = r % 16;
+    const T v = static_cast<const T *>(b == 0 ? op.P1 : op.P2)[r];
+    sP[b][c][zx] = v;                                // row-major P[z][x]
+    sP[b][c][16 + (zx % 4) * 4 + zx / 4] = v;        // column x at 16 + 4x
+  }
+  __syncthreads();
+  for (int t = threadIdx.x; t < 2 * C * 4; t += blockDim.x) {
+    const int b = t / (C * 4), r = t % (C * 4), c = r / 4, z = r % 4;
+    const T *row = &sP[b][c][z * 4];
+    sP[b][c][32 + z] = row[0] + row[1] + row[2] + row[3];  // "column 4" = row sums
+  }
+  __syncthreads();
+}
 
 template <typename T>
 __device__ inline void tip_column(const T *P, unsigned st, T (&v)[4]) {
-#pragma unroll
-  for (int z = 0; z < 4; ++z) v[z] = P[st < 4u ? z * 4 + (int)st : 16 + z];
+  V4<T>::lds(P + 16 + 4 * (st < 4u ? st : 4u), v);
 }
 
 template <typename T>
@@ -136,33 +154,40 @@ __device__ inline void matvec(const T *P, const T (&L)[4], T (&v)[4]) {
   }
 }
 
+// Rescale + store of one item (pattern `pat`, category `cat`).  All lanes of
+// the warp must call it (shuffles).  `cum_a`, `cum_b`: children's cumulative
+// exponents (already fetched), 0 when absent.
+template <typename T, int C>
+__device__ inline void finish_item(const DevOp &op, T (&r)[4], bool valid, unsigned pat, int cat,
+                                   int cum_a, int cum_b, T *out_item) {
+  if (op.scale_out != nullptr) {
+    T m = valid ? fmax(fmax(r[0], r[1]), fmax(r[2], r[3])) : T(0);
+#pragma unroll
+    for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+    const int e = frexp_exp(m);
+    if (e != 0) scale_pow2(r, e);
+    if (valid && cat == 0) op.scale_out[pat] = e + cum_a + cum_b;
+  } else if (op.scale_in != nullptr) {
+    const int e = valid ? __ldg(op.scale_in + pat) : 0;
+    if (e != 0) scale_pow2(r, e);
+  }
+  if (valid) V4<T>::st(out_item, r);
+}
+
 __device__ inline void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ inline void pdl_launch() { asm volatile("griddepcontrol.launch_dependents;" :::); }
 
+// ============================================================ latency path
 template <typename T, int C, int U>
 __global__ void __launch_bounds__(kThreads)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
-  __shared__ __align__(16) T sP[2][C][kPStride];
+  __shared__ __align__(16) T sP[2][C][kPTab];
   const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
-  const int flags = op.flags;
-  const bool tip1 = flags & OP_TIP1, tip2 = flags & OP_TIP2;
+  const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
 
-  // Everything above overlaps the previous level set; below reads its outputs.
-  pdl_wait();
+  pdl_wait();  // everything above overlaps the previous level set
   pdl_launch();
-
-  if (threadIdx.x < 2 * C * 16) {
-    const int b = threadIdx.x / (C * 16), r = threadIdx.x % (C * 16);
-    const T *src = static_cast<const T *>(b == 0 ? op.P1 : op.P2);
-    sP[b][r / 16][r % 16] = src[r];
-  }
-  __syncthreads();
-  if (threadIdx.x < 2 * C * 4) {
-    const int b = threadIdx.x / (C * 4), r = threadIdx.x % (C * 4), c = r / 4, z = r % 4;
-    const T *row = &sP[b][c][z * 4];
-    sP[b][c][16 + z] = row[0] + row[1] + row[2] + row[3];
-  }
-  __syncthreads();
+  load_ptables<T, C>(sP, op);
 
   const int cat = threadIdx.x % C;  // kThreads is a multiple of C
   const T *P1 = &sP[0][cat][0];
@@ -210,33 +235,156 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
       if (tip2) tip_column(P2, s2[j], v2); else matvec(P2, L2[j], v2);
 #pragma unroll
       for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
-      if (op.scale_out != nullptr) {
-        T m = valid ? fmax(fmax(r[0], r[1]), fmax(r[2], r[3])) : T(0);
-#pragma unroll
-        for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
-        const int e = frexp_exp(m);
-        if (e != 0) scale_pow2(r, e);
-        if (valid && cat == 0) {
-          int tot = e;
-          if (op.cum1 != nullptr) tot += __ldg(op.cum1 + pat);
-          if (op.cum2 != nullptr) tot += __ldg(op.cum2 + pat);
-          op.scale_out[pat] = tot;
-        }
-      } else if (op.scale_in != nullptr) {
-        const int e = valid ? __ldg(op.scale_in + pat) : 0;
-        if (e != 0) scale_pow2(r, e);
+      int ca = 0, cb = 0;
+      if (op.scale_out != nullptr && valid && cat == 0) {
+        if (op.cum1 != nullptr) ca = __ldg(op.cum1 + pat);
+        if (op.cum2 != nullptr) cb = __ldg(op.cum2 + pat);
       }
-      if (valid) V4<T>::st(out + (size_t)item * 4, r);
+      finish_item<T, C>(op, r, valid, pat, cat, ca, cb, out + (size_t)item * 4);
     }
   }
 }
 
+// ============================================================ bandwidth path
+__device__ inline uint32_t smem_u32(const void *p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ inline void mbar_init(uint64_t *bar, unsigned count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+__device__ inline void mbar_expect_tx(uint64_t *bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+               : "memory");
+}
+__device__ inline void mbar_wait(uint64_t *bar, unsigned parity) {
+  asm volatile(
+      "{\n.reg .pred P1;\nWAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra WAIT_%=;\n}\n" ::"r"(smem_u32(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ inline void bulk_g2s(void *dst, const void *src, unsigned bytes, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
 template <typename T, int C>
-int launch_t(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
+struct BulkStage {
+  static constexpr int kPat = kChunkItems / C;                      // patterns per chunk
+  static constexpr int kPartBytes = kChunkItems * 4 * (int)sizeof(T);
+  T c1[kChunkItems * 4];   // child-1 partials, or its tip states (kPat bytes)
+  T c2[kChunkItems * 4];
+  int32_t e1[kPat];        // child cumulative exponents (cumulative scaling)
+  int32_t e2[kPat];
+};
+
+// Issue every bulk copy of flattened chunk f into `st`, arming `bar`.
+template <typename T, int C>
+__device__ inline void issue_chunk(const DevOp *ops, int f, int nchunks, BulkStage<T, C> *st,
+                                   uint64_t *bar) {
+  using S = BulkStage<T, C>;
+  const DevOp &op = ops[f / nchunks];
+  const int chunk = f % nchunks;
+  const bool t1 = op.flags & OP_TIP1, t2 = op.flags & OP_TIP2;
+  const bool cum = op.scale_out != nullptr;
+  const bool e1 = cum && op.cum1 != nullptr, e2 = cum && op.cum2 != nullptr;
+  const unsigned b1 = t1 ? S::kPat : S::kPartBytes, b2 = t2 ? S::kPat : S::kPartBytes;
+  const unsigned be = S::kPat * 4;
+  mbar_expect_tx(bar, b1 + b2 + (e1 ? be : 0u) + (e2 ? be : 0u));
+  const size_t pat0 = (size_t)chunk * S::kPat;
+  bulk_g2s(st->c1, t1 ? (const void *)(static_cast<const uint8_t *>(op.in1) + pat0)
+                      : (const void *)(static_cast<const char *>(op.in1) + (size_t)chunk * S::kPartBytes),
+           b1, bar);
+  bulk_g2s(st->c2, t2 ? (const void *)(static_cast<const uint8_t *>(op.in2) + pat0)
+                      : (const void *)(static_cast<const char *>(op.in2) + (size_t)chunk * S::kPartBytes),
+           b2, bar);
+  if (e1) bulk_g2s(st->e1, op.cum1 + pat0, be, bar);
+  if (e2) bulk_g2s(st->e2, op.cum2 + pat0, be, bar);
+}
+
+template <typename T, int C, int kStages>
+__global__ void __launch_bounds__(kThreads)
+k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total) {
+  using S = BulkStage<T, C>;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  S *stages = reinterpret_cast<S *>(smem_raw);
+  __shared__ __align__(16) T sP[2][C][kPTab];
+  __shared__ __align__(8) uint64_t full[kStages];
+
+  const int lo = (int)((long long)total * blockIdx.x / gridDim.x);
+  const int hi = (int)((long long)total * (blockIdx.x + 1) / gridDim.x);
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  pdl_wait();  // barrier setup overlaps the previous level set
+  pdl_launch();
+  if (threadIdx.x == 0)
+    for (int s = 0; s < kStages && lo + s < hi; ++s) issue_chunk<T, C>(ops, lo + s, nchunks, &stages[s], &full[s]);
+
+  const int cat = threadIdx.x % C;
+  const unsigned nitems = (unsigned)p * C;
+  int cur = -1;
+  for (int f = lo, i = 0; f < hi; ++f, ++i) {
+    const int oi = f / nchunks, chunk = f % nchunks;
+    if (oi != cur) {  // block-uniform: new operation -> new transition tables
+      __syncthreads();
+      load_ptables<T, C>(sP, ops[oi]);
+      cur = oi;
+    }
+    const DevOp &op = ops[oi];
+    const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
+    const int s = i % kStages;
+    mbar_wait(&full[s], (unsigned)(i / kStages) & 1u);
+    const S &st = stages[s];
+    const T *P1 = &sP[0][cat][0];
+    const T *P2 = &sP[1][cat][0];
+    T *__restrict__ out = static_cast<T *>(op.out);
+#pragma unroll
+    for (int j = 0; j < kChunkItems / kThreads; ++j) {
+      const int li = threadIdx.x + j * kThreads;          // item within chunk
+      const unsigned item = (unsigned)chunk * kChunkItems + li;
+      const bool valid = item < nitems;
+      const unsigned pat = item / C;
+      const int lp = li / C;                              // pattern within chunk
+      T v1[4], v2[4], r[4];
+      if (tip1) {
+        tip_column(P1, reinterpret_cast<const uint8_t *>(st.c1)[lp], v1);
+      } else {
+        T L[4];
+        V4<T>::lds(st.c1 + li * 4, L);
+        matvec(P1, L, v1);
+      }
+      if (tip2) {
+        tip_column(P2, reinterpret_cast<const uint8_t *>(st.c2)[lp], v2);
+      } else {
+        T L[4];
+        V4<T>::lds(st.c2 + li * 4, L);
+        matvec(P2, L, v2);
+      }
+#pragma unroll
+      for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+      const int ca = (op.scale_out != nullptr && op.cum1 != nullptr) ? st.e1[lp] : 0;
+      const int cb = (op.scale_out != nullptr && op.cum2 != nullptr) ? st.e2[lp] : 0;
+      finish_item<T, C>(op, r, valid, pat, cat, ca, cb, out + (size_t)item * 4);
+    }
+    __syncthreads();  // every thread is done with stage s
+    if (threadIdx.x == 0 && f + kStages < hi)
+      issue_chunk<T, C>(ops, f + kStages, nchunks, &stages[s], &full[s]);
+  }
+}
+
+// ============================================================ host launchers
+template <typename T, int C>
+int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
   constexpr int U = 2;
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads * U - 1) / (kThreads * U));
-  // ~8 resident blocks' worth of waves over 148 SMs, at least one chunk per block
   const int target = 148 * 4 * 4;
   int gx = (target + nops - 1) / nops;
   if (gx > nchunks) gx = nchunks;
@@ -252,7 +400,6 @@ int launch_t(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(gx, ny);
     cfg.blockDim = dim3(kThreads);
-    cfg.dynamicSmemBytes = 0;
     cfg.stream = st;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -262,7 +409,54 @@ int launch_t(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream
     cudaError_t e = cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U>, pack, p, nchunks);
     if (e != cudaSuccess) return (int)e;
   }
-  return (int)cudaGetLastError();
+  return 0;
+}
+
+template <typename T, int C>
+int launch_bulk(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
+  constexpr int kStages = sizeof(T) == 4 ? 4 : 3;
+  const int nchunks = (int)(((long long)p * C + kChunkItems - 1) / kChunkItems);
+  const long long total = (long long)nops * nchunks;
+  if (total > 0x7fffffffLL) return (int)cudaErrorInvalidValue;
+  const size_t smem = sizeof(BulkStage<T, C>) * kStages;
+  static int per_sm = -1;  // per template instance
+  static int nsm = 0;
+  if (per_sm < 0) {
+    cudaError_t e = cudaFuncSetAttribute(k_partials_nuc_bulk<T, C, kStages>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return (int)e;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_bulk<T, C, kStages>,
+                                                      kThreads, smem);
+    if (e != cudaSuccess) return (int)e;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    if (per_sm < 1) per_sm = 1;
+  }
+  long long blocks = (long long)nsm * per_sm;
+  if (blocks > total) blocks = total;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)blocks);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_bulk<T, C, kStages>, d_ops, p, nchunks, (int)total);
+}
+
+// Bandwidth path once an operation has enough patterns to keep a pipeline
+// busy; the latency path for narrow work (few patterns) where a launch is
+// dominated by its fixed cost.
+constexpr long long kBulkMinItems = 64LL * 1024;
+
+template <typename T, int C>
+int launch_t(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
+  if ((long long)p * C >= kBulkMinItems) return launch_bulk<T, C>(d_ops, nops, p, st);
+  return launch_latency<T, C>(d_ops, h_ops, nops, p, st);
 }
 
 template <typename T>
