@@ -282,16 +282,15 @@ struct BulkStage {
   int32_t e2[kPat];
 };
 
-// Issue every bulk copy of flattened chunk f into `st`, arming `bar`.
+// Issue every bulk copy of chunk `chunk` of operation `oi` into `st`, arming `bar`.
 template <typename T, int C>
-__device__ inline void issue_chunk(const DevOp *ops, int f, int nchunks, BulkStage<T, C> *st,
+__device__ inline void issue_chunk(const DevOp *ops, int oi, int chunk, BulkStage<T, C> *st,
                                    uint64_t *bar) {
   using S = BulkStage<T, C>;
-  const DevOp &op = ops[f / nchunks];
-  const int chunk = f % nchunks;
+  const DevOp &op = ops[oi];
   const bool t1 = op.flags & OP_TIP1, t2 = op.flags & OP_TIP2;
   const bool cum = op.scale_out != nullptr;
-  const bool e1 = cum && op.cum1 != nullptr, e2 = cum && op.cum2 != nullptr;
+  const bool e1 = cum && !t1 && op.cum1 != nullptr, e2 = cum && !t2 && op.cum2 != nullptr;
   const unsigned b1 = t1 ? S::kPat : S::kPartBytes, b2 = t2 ? S::kPat : S::kPartBytes;
   const unsigned be = S::kPat * 4;
   mbar_expect_tx(bar, b1 + b2 + (e1 ? be : 0u) + (e2 ? be : 0u));
@@ -306,6 +305,72 @@ __device__ inline void issue_chunk(const DevOp *ops, int f, int nchunks, BulkSta
   if (e2) bulk_g2s(st->e2, op.cum2 + pat0, be, bar);
 }
 
+template <typename T, int C, int kStages, bool TIP1, bool TIP2, int SCALE>
+__device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (&P2)[16],
+                                   const T *P1tab, const T *P2tab, BulkStage<T, C> *stages,
+                                   uint64_t *full, int c0, int c1, int &i, int &pf, int &pop,
+                                   int &pchunk, int hi, int nchunks, const DevOp *ops,
+                                   unsigned nitems) {
+  const int cat = threadIdx.x % C;
+  T *__restrict__ out = static_cast<T *>(op.out);
+  for (int chunk = c0; chunk < c1; ++chunk, ++i) {
+    const int s = i % kStages;
+    mbar_wait(&full[s], (unsigned)(i / kStages) & 1u);
+    const BulkStage<T, C> &st = stages[s];
+#pragma unroll
+    for (int j = 0; j < kChunkItems / kThreads; ++j) {
+      const int li = threadIdx.x + j * kThreads;   // item within chunk
+      const int lp = li / C;                       // pattern within chunk
+      const unsigned item = (unsigned)chunk * kChunkItems + li;
+      const bool valid = item < nitems;
+      T v1[4], v2[4], r[4];
+      if (TIP1) {
+        tip_column(P1tab, reinterpret_cast<const uint8_t *>(st.c1)[lp], v1);
+      } else {
+        T L[4];
+        V4<T>::lds(st.c1 + li * 4, L);
+#pragma unroll
+        for (int z = 0; z < 4; ++z)
+          v1[z] = fma(P1[z * 4 + 3], L[3], fma(P1[z * 4 + 2], L[2], fma(P1[z * 4 + 1], L[1], P1[z * 4] * L[0])));
+      }
+      if (TIP2) {
+        tip_column(P2tab, reinterpret_cast<const uint8_t *>(st.c2)[lp], v2);
+      } else {
+        T L[4];
+        V4<T>::lds(st.c2 + li * 4, L);
+#pragma unroll
+        for (int z = 0; z < 4; ++z)
+          v2[z] = fma(P2[z * 4 + 3], L[3], fma(P2[z * 4 + 2], L[2], fma(P2[z * 4 + 1], L[1], P2[z * 4] * L[0])));
+      }
+#pragma unroll
+      for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+      if (SCALE == 1) {
+        T m = fmax(fmax(r[0], r[1]), fmax(r[2], r[3]));
+#pragma unroll
+        for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+        const int e = frexp_exp(m);
+        scale_pow2(r, e);
+        if (valid && cat == 0) {
+          int tot = e;
+          if (!TIP1 && op.cum1 != nullptr) tot += st.e1[lp];
+          if (!TIP2 && op.cum2 != nullptr) tot += st.e2[lp];
+          op.scale_out[item / C] = tot;
+        }
+      } else if (SCALE == 2) {
+        const int e = valid ? __ldg(op.scale_in + item / C) : 0;
+        scale_pow2(r, e);
+      }
+      if (valid) V4<T>::st(out + (size_t)item * 4, r);
+    }
+    __syncthreads();  // every thread is done with stage s
+    if (threadIdx.x == 0 && pf < hi) {
+      issue_chunk<T, C>(ops, pop, pchunk, &stages[s], &full[s]);
+      ++pf;
+      if (++pchunk == nchunks) { pchunk = 0; ++pop; }
+    }
+  }
+}
+
 template <typename T, int C, int kStages>
 __global__ void __launch_bounds__(kThreads)
 k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total) {
@@ -317,6 +382,7 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
 
   const int lo = (int)((long long)total * blockIdx.x / gridDim.x);
   const int hi = (int)((long long)total * (blockIdx.x + 1) / gridDim.x);
+  if (lo >= hi) return;
   if (threadIdx.x == 0) {
     for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -324,58 +390,52 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
   __syncthreads();
   pdl_wait();  // barrier setup overlaps the previous level set
   pdl_launch();
+  // producer cursor (thread 0): next flattened chunk to stream in
+  int pf = lo, pop = lo / nchunks, pchunk = lo % nchunks;
   if (threadIdx.x == 0)
-    for (int s = 0; s < kStages && lo + s < hi; ++s) issue_chunk<T, C>(ops, lo + s, nchunks, &stages[s], &full[s]);
+    for (int s = 0; s < kStages && pf < hi; ++s) {
+      issue_chunk<T, C>(ops, pop, pchunk, &stages[s], &full[s]);
+      ++pf;
+      if (++pchunk == nchunks) { pchunk = 0; ++pop; }
+    }
 
   const int cat = threadIdx.x % C;
   const unsigned nitems = (unsigned)p * C;
-  int cur = -1;
-  for (int f = lo, i = 0; f < hi; ++f, ++i) {
-    const int oi = f / nchunks, chunk = f % nchunks;
-    if (oi != cur) {  // block-uniform: new operation -> new transition tables
-      __syncthreads();
-      load_ptables<T, C>(sP, ops[oi]);
-      cur = oi;
-    }
-    const DevOp &op = ops[oi];
-    const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
-    const int s = i % kStages;
-    mbar_wait(&full[s], (unsigned)(i / kStages) & 1u);
-    const S &st = stages[s];
-    const T *P1 = &sP[0][cat][0];
-    const T *P2 = &sP[1][cat][0];
-    T *__restrict__ out = static_cast<T *>(op.out);
+  const int op_lo = lo / nchunks, op_hi = (hi - 1) / nchunks;
+  int i = 0;
+  for (int oi = op_lo; oi <= op_hi; ++oi) {
+    const int c0 = (oi == op_lo) ? lo % nchunks : 0;
+    const int c1 = (oi == op_hi) ? (hi - 1) % nchunks + 1 : nchunks;
+    __syncthreads();
+    const DevOp op = ops[oi];
+    load_ptables<T, C>(sP, op);
+    T P1[16], P2[16];
 #pragma unroll
-    for (int j = 0; j < kChunkItems / kThreads; ++j) {
-      const int li = threadIdx.x + j * kThreads;          // item within chunk
-      const unsigned item = (unsigned)chunk * kChunkItems + li;
-      const bool valid = item < nitems;
-      const unsigned pat = item / C;
-      const int lp = li / C;                              // pattern within chunk
-      T v1[4], v2[4], r[4];
-      if (tip1) {
-        tip_column(P1, reinterpret_cast<const uint8_t *>(st.c1)[lp], v1);
-      } else {
-        T L[4];
-        V4<T>::lds(st.c1 + li * 4, L);
-        matvec(P1, L, v1);
-      }
-      if (tip2) {
-        tip_column(P2, reinterpret_cast<const uint8_t *>(st.c2)[lp], v2);
-      } else {
-        T L[4];
-        V4<T>::lds(st.c2 + li * 4, L);
-        matvec(P2, L, v2);
-      }
-#pragma unroll
-      for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
-      const int ca = (op.scale_out != nullptr && op.cum1 != nullptr) ? st.e1[lp] : 0;
-      const int cb = (op.scale_out != nullptr && op.cum2 != nullptr) ? st.e2[lp] : 0;
-      finish_item<T, C>(op, r, valid, pat, cat, ca, cb, out + (size_t)item * 4);
+    for (int k = 0; k < 16; ++k) { P1[k] = sP[0][cat][k]; P2[k] = sP[1][cat][k]; }
+    const T *P1t = &sP[0][cat][0];
+    const T *P2t = &sP[1][cat][0];
+    const int scale = op.scale_out != nullptr ? 1 : (op.scale_in != nullptr ? 2 : 0);
+    const int kind = (op.flags & 3) * 3 + scale;
+#define RRL_BULK_CASE(K, T1, T2, SC)                                                            \
+  case K:                                                                                      \
+    bulk_chunks<T, C, kStages, T1, T2, SC>(op, P1, P2, P1t, P2t, stages, full, c0, c1, i, pf, pop, \
+                                           pchunk, hi, nchunks, ops, nitems);                  \
+    break;
+    switch (kind) {
+      RRL_BULK_CASE(0, false, false, 0)
+      RRL_BULK_CASE(1, false, false, 1)
+      RRL_BULK_CASE(2, false, false, 2)
+      RRL_BULK_CASE(3, true, false, 0)
+      RRL_BULK_CASE(4, true, false, 1)
+      RRL_BULK_CASE(5, true, false, 2)
+      RRL_BULK_CASE(6, false, true, 0)
+      RRL_BULK_CASE(7, false, true, 1)
+      RRL_BULK_CASE(8, false, true, 2)
+      RRL_BULK_CASE(9, true, true, 0)
+      RRL_BULK_CASE(10, true, true, 1)
+      RRL_BULK_CASE(11, true, true, 2)
     }
-    __syncthreads();  // every thread is done with stage s
-    if (threadIdx.x == 0 && f + kStages < hi)
-      issue_chunk<T, C>(ops, f + kStages, nchunks, &stages[s], &full[s]);
+#undef RRL_BULK_CASE
   }
 }
 
