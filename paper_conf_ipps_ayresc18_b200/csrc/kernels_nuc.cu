@@ -305,11 +305,41 @@ __device__ inline void issue_chunk(const DevOp *ops, int oi, int chunk, BulkStag
   if (e2) bulk_g2s(st->e2, op.cum2 + pat0, be, bar);
 }
 
+__device__ inline void mbar_arrive(uint64_t *bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+__device__ inline void consumer_sync() {  // named barrier 1: the kThreads consumer threads only
+  asm volatile("bar.sync 1, %0;" ::"n"(kThreads) : "memory");
+}
+
+// Transition tables for the consumers only (named barrier; the producer warp
+// never touches them).
+template <typename T, int C>
+__device__ inline void load_ptables_consumers(T (*sP)[C][kPTab], const DevOp &op) {
+  for (int t = threadIdx.x; t < 2 * C * 16; t += kThreads) {
+    const int b = t / (C * 16), r = t % (C * 16), c = r / 16, zx = r % 16;
+    const T v = static_cast<const T *>(b == 0 ? op.P1 : op.P2)[r];
+    sP[b][c][zx] = v;
+    sP[b][c][16 + (zx % 4) * 4 + zx / 4] = v;
+  }
+  consumer_sync();
+  for (int t = threadIdx.x; t < 2 * C * 4; t += kThreads) {
+    const int b = t / (C * 4), r = t % (C * 4), c = r / 4, z = r % 4;
+    const T *row = &sP[b][c][z * 4];
+    sP[b][c][32 + z] = row[0] + row[1] + row[2] + row[3];
+  }
+  consumer_sync();
+}
+
+// Consumer loop over chunks [c0, c1) of one operation, specialised on the
+// operation's shape (tip / internal children, scaling) so the per-item body
+// is branch-free: 2 LDS.128 (or 1 per tip child), the 4x4 mat-vecs from
+// registers, the rescale and one STG.128.  Each warp releases a stage to the
+// producer (empty barrier) as soon as it has read it.
 template <typename T, int C, int kStages, bool TIP1, bool TIP2, int SCALE>
 __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (&P2)[16],
                                    const T *P1tab, const T *P2tab, BulkStage<T, C> *stages,
-                                   uint64_t *full, int c0, int c1, int &i, int &pf, int &pop,
-                                   int &pchunk, int hi, int nchunks, const DevOp *ops,
+                                   uint64_t *full, uint64_t *empty, int c0, int c1, int &i,
                                    unsigned nitems) {
   const int cat = threadIdx.x % C;
   T *__restrict__ out = static_cast<T *>(op.out);
@@ -317,88 +347,111 @@ __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (
     const int s = i % kStages;
     mbar_wait(&full[s], (unsigned)(i / kStages) & 1u);
     const BulkStage<T, C> &st = stages[s];
+    T r[kChunkItems / kThreads][4];
+    int ex[kChunkItems / kThreads];
 #pragma unroll
-    for (int j = 0; j < kChunkItems / kThreads; ++j) {
-      const int li = threadIdx.x + j * kThreads;   // item within chunk
-      const int lp = li / C;                       // pattern within chunk
-      const unsigned item = (unsigned)chunk * kChunkItems + li;
-      const bool valid = item < nitems;
-      T v1[4], v2[4], r[4];
+    for (int j = 0; j < kChunkItems / kThreads; ++j) {  // ---- read the stage
+      const int li = threadIdx.x + j * kThreads;
+      const int lp = li / C;
+      T v1[4], v2[4];
       if (TIP1) {
         tip_column(P1tab, reinterpret_cast<const uint8_t *>(st.c1)[lp], v1);
       } else {
         T L[4];
         V4<T>::lds(st.c1 + li * 4, L);
+        if constexpr (sizeof(T) == 8) {  // fp64: rows from shared memory (register budget)
+          matvec(P1tab, L, v1);
+        } else {
 #pragma unroll
-        for (int z = 0; z < 4; ++z)
-          v1[z] = fma(P1[z * 4 + 3], L[3], fma(P1[z * 4 + 2], L[2], fma(P1[z * 4 + 1], L[1], P1[z * 4] * L[0])));
+          for (int z = 0; z < 4; ++z)
+            v1[z] = fma(P1[z * 4 + 3], L[3], fma(P1[z * 4 + 2], L[2], fma(P1[z * 4 + 1], L[1], P1[z * 4] * L[0])));
+        }
       }
       if (TIP2) {
         tip_column(P2tab, reinterpret_cast<const uint8_t *>(st.c2)[lp], v2);
       } else {
         T L[4];
         V4<T>::lds(st.c2 + li * 4, L);
+        if constexpr (sizeof(T) == 8) {  // fp64: rows from shared memory (register budget)
+          matvec(P2tab, L, v2);
+        } else {
 #pragma unroll
-        for (int z = 0; z < 4; ++z)
-          v2[z] = fma(P2[z * 4 + 3], L[3], fma(P2[z * 4 + 2], L[2], fma(P2[z * 4 + 1], L[1], P2[z * 4] * L[0])));
+          for (int z = 0; z < 4; ++z)
+            v2[z] = fma(P2[z * 4 + 3], L[3], fma(P2[z * 4 + 2], L[2], fma(P2[z * 4 + 1], L[1], P2[z * 4] * L[0])));
+        }
       }
 #pragma unroll
-      for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+      for (int z = 0; z < 4; ++z) r[j][z] = v1[z] * v2[z];
+      ex[j] = 0;
+      if (SCALE == 1 && cat == 0) {
+        if (!TIP1 && op.cum1 != nullptr) ex[j] += st.e1[lp];
+        if (!TIP2 && op.cum2 != nullptr) ex[j] += st.e2[lp];
+      }
+    }
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) mbar_arrive(&empty[s]);  // stage s free for the producer
+#pragma unroll
+    for (int j = 0; j < kChunkItems / kThreads; ++j) {  // ---- rescale + store
+      const int li = threadIdx.x + j * kThreads;
+      const unsigned item = (unsigned)chunk * kChunkItems + li;
+      const bool valid = item < nitems;
       if (SCALE == 1) {
-        T m = fmax(fmax(r[0], r[1]), fmax(r[2], r[3]));
+        T m = fmax(fmax(r[j][0], r[j][1]), fmax(r[j][2], r[j][3]));
 #pragma unroll
         for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
         const int e = frexp_exp(m);
-        scale_pow2(r, e);
-        if (valid && cat == 0) {
-          int tot = e;
-          if (!TIP1 && op.cum1 != nullptr) tot += st.e1[lp];
-          if (!TIP2 && op.cum2 != nullptr) tot += st.e2[lp];
-          op.scale_out[item / C] = tot;
-        }
+        scale_pow2(r[j], e);
+        if (valid && cat == 0) op.scale_out[item / C] = e + ex[j];
       } else if (SCALE == 2) {
         const int e = valid ? __ldg(op.scale_in + item / C) : 0;
-        scale_pow2(r, e);
+        scale_pow2(r[j], e);
       }
-      if (valid) V4<T>::st(out + (size_t)item * 4, r);
-    }
-    __syncthreads();  // every thread is done with stage s
-    if (threadIdx.x == 0 && pf < hi) {
-      issue_chunk<T, C>(ops, pop, pchunk, &stages[s], &full[s]);
-      ++pf;
-      if (++pchunk == nchunks) { pchunk = 0; ++pop; }
+      if (valid) V4<T>::st(out + (size_t)item * 4, r[j]);
     }
   }
 }
 
+// Warp-specialised persistent kernel: warps 0..7 compute, warp 8 (one elected
+// lane) streams chunks in with cp.async.bulk.  full[s]: bytes landed (tx
+// count); empty[s]: all 8 consumer warps have read stage s.
 template <typename T, int C, int kStages>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads + 32, sizeof(T) == 4 ? 3 : 2)
 k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total) {
   using S = BulkStage<T, C>;
   extern __shared__ __align__(128) unsigned char smem_raw[];
   S *stages = reinterpret_cast<S *>(smem_raw);
   __shared__ __align__(16) T sP[2][C][kPTab];
   __shared__ __align__(8) uint64_t full[kStages];
+  __shared__ __align__(8) uint64_t empty[kStages];
 
   const int lo = (int)((long long)total * blockIdx.x / gridDim.x);
   const int hi = (int)((long long)total * (blockIdx.x + 1) / gridDim.x);
   if (lo >= hi) return;
-  if (threadIdx.x == 0) {
-    for (int s = 0; s < kStages; ++s) mbar_init(&full[s], 1);
+  if (threadIdx.x == kThreads) {
+    for (int s = 0; s < kStages; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&empty[s], kThreads / 32);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   __syncthreads();
   pdl_wait();  // barrier setup overlaps the previous level set
   pdl_launch();
-  // producer cursor (thread 0): next flattened chunk to stream in
-  int pf = lo, pop = lo / nchunks, pchunk = lo % nchunks;
-  if (threadIdx.x == 0)
-    for (int s = 0; s < kStages && pf < hi; ++s) {
-      issue_chunk<T, C>(ops, pop, pchunk, &stages[s], &full[s]);
-      ++pf;
-      if (++pchunk == nchunks) { pchunk = 0; ++pop; }
-    }
 
+  if (threadIdx.x >= kThreads) {  // ------------------------------ producer warp
+    if (threadIdx.x == kThreads) {
+      int oi = lo / nchunks, chunk = lo % nchunks;
+      for (int k = 0, f = lo; f < hi; ++f, ++k) {
+        const int s = k % kStages;
+        mbar_wait(&empty[s], ((unsigned)(k / kStages) & 1u) ^ 1u);
+        issue_chunk<T, C>(ops, oi, chunk, &stages[s], &full[s]);
+        if (++chunk == nchunks) { chunk = 0; ++oi; }
+      }
+    }
+    return;
+  }
+
+  // ------------------------------------------------------------------ consumers
   const int cat = threadIdx.x % C;
   const unsigned nitems = (unsigned)p * C;
   const int op_lo = lo / nchunks, op_hi = (hi - 1) / nchunks;
@@ -406,9 +459,9 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
   for (int oi = op_lo; oi <= op_hi; ++oi) {
     const int c0 = (oi == op_lo) ? lo % nchunks : 0;
     const int c1 = (oi == op_hi) ? (hi - 1) % nchunks + 1 : nchunks;
-    __syncthreads();
+    consumer_sync();  // previous op's tables no longer in use
     const DevOp op = ops[oi];
-    load_ptables<T, C>(sP, op);
+    load_ptables_consumers<T, C>(sP, op);
     T P1[16], P2[16];
 #pragma unroll
     for (int k = 0; k < 16; ++k) { P1[k] = sP[0][cat][k]; P2[k] = sP[1][cat][k]; }
@@ -416,10 +469,10 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
     const T *P2t = &sP[1][cat][0];
     const int scale = op.scale_out != nullptr ? 1 : (op.scale_in != nullptr ? 2 : 0);
     const int kind = (op.flags & 3) * 3 + scale;
-#define RRL_BULK_CASE(K, T1, T2, SC)                                                            \
-  case K:                                                                                      \
-    bulk_chunks<T, C, kStages, T1, T2, SC>(op, P1, P2, P1t, P2t, stages, full, c0, c1, i, pf, pop, \
-                                           pchunk, hi, nchunks, ops, nitems);                  \
+#define RRL_BULK_CASE(K, T1, T2, SC)                                                               \
+  case K:                                                                                         \
+    bulk_chunks<T, C, kStages, T1, T2, SC>(op, P1, P2, P1t, P2t, stages, full, empty, c0, c1, i,   \
+                                           nitems);                                               \
     break;
     switch (kind) {
       RRL_BULK_CASE(0, false, false, 0)
@@ -486,7 +539,7 @@ int launch_bulk(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;
     e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_bulk<T, C, kStages>,
-                                                      kThreads, smem);
+                                                      kThreads + 32, smem);
     if (e != cudaSuccess) return (int)e;
     int dev = 0;
     cudaGetDevice(&dev);
@@ -497,7 +550,7 @@ int launch_bulk(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   if (blocks > total) blocks = total;
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3((unsigned)blocks);
-  cfg.blockDim = dim3(kThreads);
+  cfg.blockDim = dim3(kThreads + 32);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute at[1];
