@@ -231,6 +231,8 @@ def main():
     ap.add_argument("--impl", default="ours", choices=("ours", "reference"))
     ap.add_argument("--no-graph", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-secondary", action="store_true",
+                    help="skip the configs[2] HBM-regime measurement that rides along with c1")
     ap.add_argument("--ref-patterns", type=int, default=10_000)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
@@ -258,17 +260,24 @@ def main():
     _b.build()
     from paper_conf_ipps_ayresc18_b200 import TreeLikelihood, rrl as R
 
-    w, scaling = rank_workload(args.config, rank, world)
-    n, p, c, s = w.n, w.p, w.c, w.s
-    elt = 4 if args.precision == 32 else 8
     stream = torch.cuda.current_stream()
-    reuse = args.config == "c4"
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
+    d_out = torch.zeros(1, dtype=torch.float64, device="cuda")
+    peaks, peak_src = measured_peaks()
+    hbm = float(peaks.get("hbm_gbs", 6650.0))
 
-    def make(mode):
+    def maxall(x):
+        if dist is None:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def make(w, mode, precision, reuse):
         nbuf = None
         if reuse:
-            nbuf = R.rrl_reroot_and_schedule(n, w.tree.parent, w.tree.blen, mode, True)["buffer_count"]
-        tl = TreeLikelihood(n, p, s, c, precision=args.precision, device=local,
+            nbuf = R.rrl_reroot_and_schedule(w.n, w.tree.parent, w.tree.blen, mode, True)["buffer_count"]
+        tl = TreeLikelihood(w.n, w.p, w.s, w.c, precision=precision, device=local,
                             cuda_graph=not args.no_graph, buffer_count=nbuf,
                             stream_ptr=stream.cuda_stream)
         tl.set_model_params(w.model, w.rates, w.cat_weights)
@@ -277,9 +286,6 @@ def main():
         tl.set_tree(w.tree.parent, w.tree.blen, mode, reuse_buffers=reuse)
         return tl
 
-    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device="cuda")
-    d_out = torch.zeros(1, dtype=torch.float64, device="cuda")
-
     def step(tl):
         tl.update()
         tl.root_loglik_device(d_out.data_ptr())
@@ -287,6 +293,8 @@ def main():
             dist.all_reduce(d_out)
 
     def timed(tl, steps, warmup):
+        """Per-step CUDA events on the launching stream; L2 flushed before
+        every step outside the events; barrier + synchronize on both sides."""
         for _ in range(warmup):
             flush.zero_()
             step(tl)
@@ -308,14 +316,7 @@ def main():
         torch.cuda.synchronize()
         ms = sum(a.elapsed_time(b) for a, b in evs)
         launches = R.rrl_get_profile(tl.inst)["kernel_launches"]
-        return ms, launches
-
-    def maxall(x):
-        if dist is None:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
+        return maxall(ms), launches
 
     def instrumented(tl, steps):
         """Per-launch CUDA events (library profiling mode, eager launches) on
@@ -329,40 +330,69 @@ def main():
         R.rrl_set_profiling(tl.inst, False)
         return prof
 
-    # ---- rerooted (the product configuration)
-    tl = make("reroot")
-    sched = tl.sched
-    clocks = ClockSampler(local)
-    ms, launches = timed(tl, args.steps, args.warmup)
-    clk = clocks.stop()
-    ms_max = maxall(ms)
-    fl = flops_per_pass(n, p, c, s)
-    value = fl * world * args.steps / (ms_max * 1e-3) / 1e9
-    prof = instrumented(tl, min(args.steps, 100))
-    nsteps_i = min(args.steps, 100)
-    part_ms = prof["partials_ms"] / nsteps_i
-    nlaunch = prof["partials_launches"] / nsteps_i
-    bpp = bytes_per_pass(sched["ops"], n, p, c, s, elt)
-    achieved = bpp / (part_ms * 1e-3) / 1e9
-    peaks, peak_src = measured_peaks()
-    hbm = float(peaks.get("hbm_gbs", 6650.0))
-    traffic = ncu_traffic(args.config, args.precision)
-    lnl = float(d_out.item())
+    def measure(cfg, precision, steps, warmup, with_original=True, keep=False):
+        w, scaling = rank_workload(cfg, rank, world)
+        n, p, c, s = w.n, w.p, w.c, w.s
+        elt = 4 if precision == 32 else 8
+        reuse = cfg == "c4"
+        tl = make(w, "reroot", precision, reuse)
+        sched = tl.sched
+        clocks = ClockSampler(local)
+        ms, launches = timed(tl, steps, warmup)
+        clk = clocks.stop()
+        fl = flops_per_pass(n, p, c, s)
+        nsi = min(steps, 100)
+        prof = instrumented(tl, nsi)
+        part_ms = prof["partials_ms"] / nsi
+        bpp = bytes_per_pass(sched["ops"], n, p, c, s, elt)
+        achieved = bpp / (part_ms * 1e-3) / 1e9
+        res = {
+            "cfg": cfg, "w": w, "scaling": scaling, "n": n, "p": p, "c": c, "s": s,
+            "value": fl * world * steps / (ms * 1e-3) / 1e9, "ms_per_step": ms / steps,
+            "launches": launches, "clocks": clk, "sets": sched["set_count"], "fl": fl,
+            "updatePartials": {"ms_per_pass": part_ms,
+                               "launches_per_pass": prof["partials_launches"] / nsi,
+                               "gflops": fl / (part_ms * 1e-3) / 1e9,
+                               "pattern_node_updates_per_s": (n - 1) * p / (part_ms * 1e-3),
+                               "share_of_step": part_ms / (ms / steps)},
+            "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
+                         "frac": achieved / hbm, "traffic": ncu_traffic(cfg, precision),
+                         "kernel": "k_partials_nuc / k_partials_nuc_bulk (updatePartials, one "
+                                   "launch per level set)",
+                         "algorithmic_bytes_per_pass": bpp,
+                         "launches_per_pass": prof["partials_launches"] / nsi,
+                         "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json)",
+                         "timing": "per-launch CUDA events on the launching stream, eager "
+                                   f"instrumented pass of {nsi} steps after the timed region"},
+            "lnL": float(d_out.item()),
+        }
+        if with_original and cfg != "c4":
+            to = make(w, "level", precision, False)
+            ms_o, _ = timed(to, steps, warmup)
+            prof_o = instrumented(to, nsi)
+            po = prof_o["partials_ms"] / nsi
+            res["reroot"] = {
+                "sets": sched["set_count"], "sets_original": to.sched["set_count"],
+                "theoretical_speedup": to.sched["set_count"] / sched["set_count"],
+                "step_speedup": ms_o / ms, "updatePartials_speedup": po / part_ms,
+                "original_gflops": fl * world * steps / (ms_o * 1e-3) / 1e9,
+                "paper_context": "BEAGLE CUDA on Quadro GP100: up to 1.93x (pectinate, 406 OTUs, "
+                                 "512 patterns, PAPER.md:258); mean 1.26x (random 256 OTUs, "
+                                 "PAPER.md:230)"}
+            to.close()
+        if keep:
+            res["tl"] = tl
+        else:
+            tl.close()
+        return res
 
-    # ---- original rooting, same kernels (the reroot speedup of the paper)
-    orig = {}
-    if args.config != "c4":
-        to = make("level")
-        ms_o, _ = timed(to, args.steps, args.warmup)
-        ms_o = maxall(ms_o)
-        prof_o = instrumented(to, nsteps_i)
-        orig = {"sets": to.sched["set_count"], "gflops": fl * world * args.steps / (ms_o * 1e-3) / 1e9,
-                "ms_per_step": ms_o / args.steps,
-                "updatePartials_ms": prof_o["partials_ms"] / nsteps_i}
-        to.close()
+    prim = measure(args.config, args.precision, args.steps, args.warmup, keep=True)
+    w, tl = prim["w"], prim["tl"]
+    n, p = prim["n"], prim["p"]
 
     # ---- e2e through the public API with host buffers (pinned), every step:
     # reroot + schedule, H2D tips + branch lengths, pass, D2H of the lnL.
+    reuse = args.config == "c4"
     pinned = torch.empty(w.tips.shape, dtype=torch.uint8, pin_memory=True).numpy()
     pinned[:] = w.tips
     e2e_steps = max(3, min(args.steps, 50))
@@ -381,59 +411,57 @@ def main():
         tl.root_loglik_device(d_out.data_ptr())
         if dist is not None:
             dist.all_reduce(d_out)
-        host_l = float(d_out.item())
+        float(d_out.item())
     e2e_s = maxall(time.perf_counter() - t0)
-    e2e_val = fl * world * e2e_steps / e2e_s / 1e9
+    e2e_val = prim["fl"] * world * e2e_steps / e2e_s / 1e9
     h2d = int(w.tips.nbytes + tl.t.nbytes + tl.matrix_idx.nbytes)
     tl.close()
 
+    # ---- the HBM-bound regime (configs[2]) beside the launch-bound headline
+    sec = None
+    if args.config == "c1" and not args.no_secondary:
+        sec = measure("c2", args.precision, min(args.steps, 30), args.warmup)
+
     if rank != 0:
+        if dist is not None:
+            dist.destroy_process_group()
         return
     cpu = None if args.no_cpu_baseline else cpu_baseline(w)
     out = {
         "metric": METRIC,
-        "value": value,
+        "value": prim["value"],
         "unit": "GFLOPS",
         "n_gpus": world,
         "steps": args.steps,
         "warmup": args.warmup,
-        "ms_per_step": ms_max / args.steps,
+        "ms_per_step": prim["ms_per_step"],
         "higher_is_better": True,
-        "scaling": scaling,
+        "scaling": prim["scaling"],
         "vs_baseline": None,
         "dtype": f"f{args.precision}",
         "data": "synthetic (seeded workloads/: tree, GTR+G4 parameters, uniform alignment)",
         "config": {"workload": CONFIG_DESC[args.config], "n_tips": n, "patterns_per_gpu": p,
-                   "categories": c, "states": s, "schedule": "reroot", "sets": sched["set_count"],
-                   "cuda_graph": not args.no_graph,
+                   "categories": prim["c"], "states": prim["s"], "schedule": "reroot",
+                   "sets": prim["sets"], "cuda_graph": not args.no_graph,
                    "l2": "flushed before every step (512 MiB memset, outside the step events)"},
-        "reroot": {"sets": sched["set_count"], "sets_original": orig.get("sets"),
-                   "theoretical_speedup": (orig["sets"] / sched["set_count"]) if orig else None,
-                   "step_speedup": (ms_o / ms_max) if orig else None,
-                   "updatePartials_speedup": (orig["updatePartials_ms"] / part_ms) if orig else None,
-                   "original_gflops": orig.get("gflops"),
-                   "paper_context": "BEAGLE CUDA on Quadro GP100: up to 1.93x (pectinate, 406 OTUs, "
-                                    "512 patterns, PAPER.md:258); mean 1.26x (random 256 OTUs, PAPER.md:230)"},
-        "updatePartials": {"ms_per_pass": part_ms, "launches_per_pass": nlaunch,
-                           "gflops": fl / (part_ms * 1e-3) / 1e9,
-                           "pattern_node_updates_per_s": (n - 1) * p / (part_ms * 1e-3),
-                           "share_of_step": part_ms / (ms_max / args.steps)},
-        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm, "unit": "GB/s",
-                     "frac": achieved / hbm, "traffic": traffic,
-                     "kernel": "k_partials_nuc (updatePartials, one launch per level set)",
-                     "algorithmic_bytes_per_pass": bpp,
-                     "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json)",
-                     "timing": "per-launch CUDA events on the launching stream, eager "
-                               f"instrumented pass of {nsteps_i} steps after the timed region"},
+        "reroot": prim.get("reroot"),
+        "updatePartials": prim["updatePartials"],
+        "roofline": prim["roofline"],
         "cpu_baseline": cpu,
         "e2e": {"value": e2e_val, "unit": "GFLOPS", "h2d_bytes_per_step": h2d,
                 "d2h_bytes_per_step": 8, "steps": e2e_steps,
                 "path": "TreeLikelihood: set_tips (pinned H2D) + rrl_reroot_and_schedule + K1 + "
                         "level-set K2 + K4 + D2H lnL"},
-        "gpu_launches": int(launches),
-        "clocks": clk,
-        "lnL": lnl,
+        "gpu_launches": int(prim["launches"]),
+        "clocks": prim["clocks"],
+        "lnL": prim["lnL"],
     }
+    if sec is not None:
+        out["hbm_regime"] = {
+            "workload": CONFIG_DESC["c2"], "value": sec["value"], "unit": "GFLOPS",
+            "ms_per_step": sec["ms_per_step"], "reroot": sec.get("reroot"),
+            "updatePartials": sec["updatePartials"], "roofline": sec["roofline"],
+            "gpu_launches": int(sec["launches"]), "clocks": sec["clocks"]}
     print(json.dumps(out), flush=True)
     if dist is not None:
         dist.destroy_process_group()

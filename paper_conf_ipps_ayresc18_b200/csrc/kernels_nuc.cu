@@ -178,33 +178,61 @@ __device__ inline void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "mem
 __device__ inline void pdl_launch() { asm volatile("griddepcontrol.launch_dependents;" :::); }
 
 // ============================================================ latency path
+// One dependent memory round trip per launch: after griddepcontrol.wait every
+// thread issues its transition-matrix rows (L2-resident), its child vectors
+// and its children's exponents together, then computes and stores.
+template <typename T>
+__device__ inline void tip_select(const T (&P)[16], unsigned st, T (&v)[4]) {
+#pragma unroll
+  for (int z = 0; z < 4; ++z) {
+    const T rs = P[z * 4] + P[z * 4 + 1] + P[z * 4 + 2] + P[z * 4 + 3];
+    T a = (st == 0u) ? P[z * 4] : rs;
+    a = (st == 1u) ? P[z * 4 + 1] : a;
+    a = (st == 2u) ? P[z * 4 + 2] : a;
+    a = (st == 3u) ? P[z * 4 + 3] : a;
+    v[z] = a;
+  }
+}
+
+template <typename T>
+__device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
+#pragma unroll
+  for (int z = 0; z < 4; ++z)
+    v[z] = fma(P[z * 4 + 3], L[3], fma(P[z * 4 + 2], L[2], fma(P[z * 4 + 1], L[1], P[z * 4] * L[0])));
+}
+
 template <typename T, int C, int U>
 __global__ void __launch_bounds__(kThreads)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
-  __shared__ __align__(16) T sP[2][C][kPTab];
   const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
-
-  pdl_wait();  // everything above overlaps the previous level set
-  pdl_launch();
-  load_ptables<T, C>(sP, op);
-
   const int cat = threadIdx.x % C;  // kThreads is a multiple of C
-  const T *P1 = &sP[0][cat][0];
-  const T *P2 = &sP[1][cat][0];
+  const T *__restrict__ P1g = static_cast<const T *>(op.P1) + cat * 16;
+  const T *__restrict__ P2g = static_cast<const T *>(op.P2) + cat * 16;
   const T *__restrict__ L1g = static_cast<const T *>(op.in1);
   const T *__restrict__ L2g = static_cast<const T *>(op.in2);
   const uint8_t *__restrict__ S1g = static_cast<const uint8_t *>(op.in1);
   const uint8_t *__restrict__ S2g = static_cast<const uint8_t *>(op.in2);
   T *__restrict__ out = static_cast<T *>(op.out);
+  const bool scale_w = op.scale_out != nullptr;
   const unsigned nitems = (unsigned)p * C;
 
+  pdl_wait();  // everything above overlaps the previous level set
+  pdl_launch();
+
+  T P1[16], P2[16];
+#pragma unroll
+  for (int k = 0; k < 16; k += 4) {
+    V4<T>::ld(P1g + k, *reinterpret_cast<T(*)[4]>(&P1[k]));
+    V4<T>::ld(P2g + k, *reinterpret_cast<T(*)[4]>(&P2[k]));
+  }
   for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
     const unsigned base = (unsigned)chunk * (kThreads * U) + threadIdx.x;
     T L1[U][4], L2[U][4];
     unsigned s1[U], s2[U];
+    int ca[U], cb[U];
 #pragma unroll
-    for (int j = 0; j < U; ++j) {  // ---- all child reads of this thread in flight together
+    for (int j = 0; j < U; ++j) {  // ---- all reads of this thread in flight together
       const unsigned item = base + j * kThreads;
       const bool valid = item < nitems;
       const unsigned pat = item / C;
@@ -224,6 +252,8 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
 #pragma unroll
         for (int z = 0; z < 4; ++z) L2[j][z] = T(0);
       }
+      ca[j] = (scale_w && valid && cat == 0 && op.cum1 != nullptr) ? __ldg(op.cum1 + pat) : 0;
+      cb[j] = (scale_w && valid && cat == 0 && op.cum2 != nullptr) ? __ldg(op.cum2 + pat) : 0;
     }
 #pragma unroll
     for (int j = 0; j < U; ++j) {  // ---- compute + store
@@ -231,16 +261,11 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
       const bool valid = item < nitems;
       const unsigned pat = item / C;
       T v1[4], v2[4], r[4];
-      if (tip1) tip_column(P1, s1[j], v1); else matvec(P1, L1[j], v1);
-      if (tip2) tip_column(P2, s2[j], v2); else matvec(P2, L2[j], v2);
+      if (tip1) tip_select(P1, s1[j], v1); else matvec_r(P1, L1[j], v1);
+      if (tip2) tip_select(P2, s2[j], v2); else matvec_r(P2, L2[j], v2);
 #pragma unroll
       for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
-      int ca = 0, cb = 0;
-      if (op.scale_out != nullptr && valid && cat == 0) {
-        if (op.cum1 != nullptr) ca = __ldg(op.cum1 + pat);
-        if (op.cum2 != nullptr) cb = __ldg(op.cum2 + pat);
-      }
-      finish_item<T, C>(op, r, valid, pat, cat, ca, cb, out + (size_t)item * 4);
+      finish_item<T, C>(op, r, valid, pat, cat, ca[j], cb[j], out + (size_t)item * 4);
     }
   }
 }
@@ -495,7 +520,7 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
 // ============================================================ host launchers
 template <typename T, int C>
 int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
-  constexpr int U = 2;
+  constexpr int U = 1;
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads * U - 1) / (kThreads * U));
   const int target = 148 * 4 * 4;
