@@ -523,8 +523,16 @@ int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cuda
   constexpr int U = 1;
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads * U - 1) / (kThreads * U));
-  const int target = 148 * 4 * 4;
-  int gx = (target + nops - 1) / nops;
+  // One wave: a second wave would double this launch's latency.
+  static int resident = -1;  // per template instance
+  if (resident < 0) {
+    int per_sm = 1, dev = 0, nsm = 148;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, U>, kThreads, 0);
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    resident = (per_sm > 0 ? per_sm : 1) * nsm;
+  }
+  int gx = resident / nops;
   if (gx > nchunks) gx = nchunks;
   if (gx < 1) gx = 1;
   for (int o = 0; o < nops; o += 65535) {
