@@ -220,12 +220,20 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
   pdl_wait();  // everything above overlaps the previous level set
   pdl_launch();
 
-  T P1[16], P2[16];
+  // fp32: each thread holds its category's rows in registers.  fp64: the rows
+  // would cost 64 registers, so the block stages the tables in shared memory
+  // (issued after this thread's first child loads, see below).
+  constexpr bool kRegP = sizeof(T) == 4;
+  __shared__ __align__(16) T sP[kRegP ? 1 : 2][kRegP ? 1 : C][kRegP ? 4 : kPTab];
+  T P1[kRegP ? 16 : 1], P2[kRegP ? 16 : 1];
+  if constexpr (kRegP) {
 #pragma unroll
-  for (int k = 0; k < 16; k += 4) {
-    V4<T>::ld(P1g + k, *reinterpret_cast<T(*)[4]>(&P1[k]));
-    V4<T>::ld(P2g + k, *reinterpret_cast<T(*)[4]>(&P2[k]));
+    for (int k = 0; k < 16; k += 4) {
+      V4<T>::ld(P1g + k, *reinterpret_cast<T(*)[4]>(&P1[k]));
+      V4<T>::ld(P2g + k, *reinterpret_cast<T(*)[4]>(&P2[k]));
+    }
   }
+  bool tables = kRegP;
   for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
     const unsigned base = (unsigned)chunk * (kThreads * U) + threadIdx.x;
     T L1[U][4], L2[U][4];
@@ -255,14 +263,26 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
       ca[j] = (scale_w && valid && cat == 0 && op.cum1 != nullptr) ? __ldg(op.cum1 + pat) : 0;
       cb[j] = (scale_w && valid && cat == 0 && op.cum2 != nullptr) ? __ldg(op.cum2 + pat) : 0;
     }
+    if constexpr (!kRegP) {
+      if (!tables) {  // block-uniform, first chunk only
+        load_ptables<T, C>(sP, op);
+        tables = true;
+      }
+    }
 #pragma unroll
     for (int j = 0; j < U; ++j) {  // ---- compute + store
       const unsigned item = base + j * kThreads;
       const bool valid = item < nitems;
       const unsigned pat = item / C;
       T v1[4], v2[4], r[4];
-      if (tip1) tip_select(P1, s1[j], v1); else matvec_r(P1, L1[j], v1);
-      if (tip2) tip_select(P2, s2[j], v2); else matvec_r(P2, L2[j], v2);
+      if constexpr (kRegP) {
+        if (tip1) tip_select(P1, s1[j], v1); else matvec_r(P1, L1[j], v1);
+        if (tip2) tip_select(P2, s2[j], v2); else matvec_r(P2, L2[j], v2);
+      } else {
+        const T *t1 = &sP[0][cat][0], *t2 = &sP[kRegP ? 0 : 1][cat][0];
+        if (tip1) tip_column(t1, s1[j], v1); else matvec(t1, L1[j], v1);
+        if (tip2) tip_column(t2, s2[j], v2); else matvec(t2, L2[j], v2);
+      }
 #pragma unroll
       for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
       finish_item<T, C>(op, r, valid, pat, cat, ca[j], cb[j], out + (size_t)item * 4);
