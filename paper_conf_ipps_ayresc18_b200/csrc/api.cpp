@@ -77,7 +77,11 @@ struct Instance {
   std::vector<rrl_op> last_ops;
   std::vector<int32_t> last_offs;
   bool ops_valid = false;
-  cudaGraphExec_t graph = nullptr;
+  cudaGraphExec_t graph = nullptr;       // replay of the set launches
+  cudaGraphExec_t graph_prof = nullptr;  // same, with an external event between sets
+  std::vector<cudaEvent_t> gev;          // events of graph_prof (nsets + 1)
+  bool gev_pending = false;
+  int gev_nsets = 0;
   cudaStream_t graph_stream = nullptr;
   int graph_kernels = 0;
 
@@ -141,7 +145,7 @@ struct Timed {  // brackets one launch with events when profiling
   Instance *I;
   EvPair ep{};
   bool on;
-  Timed(Instance *in, int kind) : I(in), on(in->profiling) {
+  Timed(Instance *in, int kind, bool enabled = true) : I(in), on(in->profiling && enabled) {
     if (on) {
       ep.a = take_event(I);
       ep.b = take_event(I);
@@ -174,10 +178,35 @@ void drain_events(Instance *I) {
   I->events.clear();
 }
 
+// Sum the per-set durations of the last profiled graph replay.
+int drain_graph_events(Instance *I) {
+  if (!I->gev_pending) return 0;
+  CK(cudaEventSynchronize(I->gev[I->gev_nsets]));
+  for (int k = 0; k < I->gev_nsets; ++k) {
+    float ms = 0.f;
+    CK(cudaEventElapsedTime(&ms, I->gev[k], I->gev[k + 1]));
+    I->prof.partials_ms += ms;
+  }
+  I->gev_pending = false;
+  return 0;
+}
+
+int drop_graphs(Instance *I) {
+  int r = drain_graph_events(I);
+  if (r < 0) return r;
+  if (I->graph) cudaGraphExecDestroy(I->graph);
+  if (I->graph_prof) cudaGraphExecDestroy(I->graph_prof);
+  I->graph = nullptr;
+  I->graph_prof = nullptr;
+  return 0;
+}
+
 void destroy(Instance *I) {
   cudaSetDevice(I->device);
   if (I->stream) cudaStreamSynchronize(I->stream);
   if (I->graph) cudaGraphExecDestroy(I->graph);
+  if (I->graph_prof) cudaGraphExecDestroy(I->graph_prof);
+  for (auto e : I->gev) cudaEventDestroy(e);
   for (void *t : I->tip_partials)
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
@@ -679,16 +708,18 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
     I->last_ops.assign(ops, ops + op_count);
     I->last_offs = offs;
     I->ops_valid = true;
-    if (I->graph) {
-      cudaGraphExecDestroy(I->graph);
-      I->graph = nullptr;
-    }
+    int rg = drop_graphs(I);
+    if (rg < 0) return rg;
   }
 
-  auto launch_all = [&]() -> int {
+  // events_in_graph: record an external event before every set launch and
+  // after the last one (profiling inside a graph replay); otherwise, when
+  // profiling eagerly, bracket each launch with its own events.
+  auto launch_all = [&](bool capturing, bool events_in_graph) -> int {
     for (int k = 0; k < nsets; ++k) {
       const int n = offs[k + 1] - offs[k];
-      Timed tm(I, 0);
+      if (events_in_graph) CK(cudaEventRecordWithFlags(I->gev[k], I->stream, cudaEventRecordExternal));
+      Timed tm(I, 0, !capturing);
       int e = (I->s == 4) ? launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k],
                                                        I->h_ops + offs[k], n, I->p, I->p_pad, I->stream)
                           : launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k],
@@ -697,44 +728,55 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
       if (e != 0) return fail(RRL_ERROR_CUDA, std::string("updatePartials launch: ") +
                                                   cudaGetErrorString(static_cast<cudaError_t>(e)));
     }
+    if (events_in_graph) CK(cudaEventRecordWithFlags(I->gev[nsets], I->stream, cudaEventRecordExternal));
     return 0;
   };
+  int kl = 0;
+  for (int k = 0; k < nsets; ++k) kl += (offs[k + 1] - offs[k] + 65534) / 65535;
 
   // (the legacy default stream cannot be captured: eager launches there)
-  const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && !I->profiling && I->stream != nullptr;
+  const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && I->stream != nullptr;
   if (use_graph) {
-    if (I->graph && I->graph_stream != I->stream) {
-      cudaGraphExecDestroy(I->graph);
-      I->graph = nullptr;
+    const bool prof = I->profiling;
+    cudaGraphExec_t &gx = prof ? I->graph_prof : I->graph;
+    if ((I->graph || I->graph_prof) && I->graph_stream != I->stream) {
+      int r = drop_graphs(I);
+      if (r < 0) return r;
     }
-    if (!I->graph) {
+    if (prof) {
+      int r = drain_graph_events(I);
+      if (r < 0) return r;
+      while ((int)I->gev.size() < nsets + 1) {
+        cudaEvent_t e;
+        CK(cudaEventCreate(&e));
+        I->gev.push_back(e);
+      }
+    }
+    if (!gx) {
       cudaGraph_t g;
       CK(cudaStreamBeginCapture(I->stream, cudaStreamCaptureModeThreadLocal));
-      int e = launch_all();
+      int e = launch_all(true, prof);
       cudaError_t ce = cudaStreamEndCapture(I->stream, &g);
       if (e < 0) return e;
       CK(ce);
-      cudaError_t ie = cudaGraphInstantiate(&I->graph, g, 0);
+      cudaError_t ie = cudaGraphInstantiate(&gx, g, 0);
       cudaGraphDestroy(g);
       CK(ie);
       I->graph_stream = I->stream;
-      size_t nn = 0;
-      I->graph_kernels = 0;
-      (void)nn;
-      for (int k = 0; k < nsets; ++k) I->graph_kernels += (offs[k + 1] - offs[k] + 65534) / 65535;
+      I->graph_kernels = kl;
     }
-    CK(cudaGraphLaunch(I->graph, I->stream));
+    CK(cudaGraphLaunch(gx, I->stream));
+    if (prof) {
+      I->gev_pending = true;
+      I->gev_nsets = nsets;
+    }
     I->prof.graph_launches += 1;
-    I->prof.kernel_launches += I->graph_kernels;
-    I->prof.partials_launches += I->graph_kernels;
   } else {
-    int e = launch_all();
+    int e = launch_all(false, false);
     if (e < 0) return e;
-    int kl = 0;
-    for (int k = 0; k < nsets; ++k) kl += (offs[k + 1] - offs[k] + 65534) / 65535;
-    I->prof.kernel_launches += kl;
-    I->prof.partials_launches += kl;
   }
+  I->prof.kernel_launches += kl;
+  I->prof.partials_launches += kl;
   return RRL_SUCCESS;
 }
 
@@ -879,6 +921,8 @@ int rrl_get_profile(int inst, rrl_profile *out) {
   if (!out) return fail(RRL_ERROR_GENERAL, "out NULL");
   CK(cudaStreamSynchronize(I->stream));
   drain_events(I);
+  int r = drain_graph_events(I);
+  if (r < 0) return r;
   *out = I->prof;
   return RRL_SUCCESS;
 }
@@ -887,6 +931,8 @@ int rrl_reset_profile(int inst) {
   GET(I, inst);
   CK(cudaStreamSynchronize(I->stream));
   drain_events(I);
+  int r = drain_graph_events(I);
+  if (r < 0) return r;
   I->prof = rrl_profile{};
   return RRL_SUCCESS;
 }

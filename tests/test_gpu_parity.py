@@ -127,6 +127,12 @@ def test_greedy_batching_and_graph_and_determinism():
     assert tg.loglik() == a and tg.loglik() == a         # graph capture, then replay
     prof = R.rrl_get_profile(tg.inst)
     assert prof["graph_launches"] == 2
+    R.rrl_set_profiling(tg.inst, True)                   # per-set events inside the graph
+    R.rrl_reset_profile(tg.inst)
+    assert tg.loglik() == a and tg.loglik() == a
+    prof = R.rrl_get_profile(tg.inst)
+    assert prof["graph_launches"] == 2 and prof["partials_ms"] > 0
+    assert prof["partials_launches"] == 2 * tg.sched["set_count"]
     tg.close()
 
 
@@ -259,6 +265,65 @@ def test_edge_loglik_pulley():
     ch = pruning.children_of(t.parent)
     a, b = ch[t.root]
     # matrix for branch a with length t_a + t_b
+    R.rrl_update_transition_matrices(tl.inst, 0, np.array([a], np.int32),
+                                     np.array([t.blen[a] + t.blen[b]]))
+    e = R.rrl_calculate_edge_log_likelihoods(tl.inst, b, a, a, 0, 0, b - w.n, a - w.n)
+    assert rel(e, root_l) <= 1e-12
+    tl.close()
+
+
+# ------------------------------------------------------------------ codon (61 states)
+@pytest.mark.parametrize("precision", [64, 32])
+def test_codon_transition_matrices(precision):
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="random", n=10, p=10, model="gy94", c=4, seed=3)
+    tl = gpu_setup(w, "level", precision)
+    tl.update()
+    Q = om.rate_matrix(w.model)
+    tol = 1e-12 if precision == 64 else 2e-7
+    for m in tl.matrix_idx[:6]:
+        got = R.rrl_get_transition_matrix(tl.inst, int(m), w.c, w.s)
+        for k in range(w.c):
+            exp = pruning.transition_matrix(Q, w.rates[k] * w.tree.blen[m])
+            np.testing.assert_allclose(got[k], exp, atol=tol, rtol=0)
+    tl.close()
+
+
+@pytest.mark.parametrize("precision", [64, 32])
+@pytest.mark.parametrize("mode", ["reroot", "level"])
+def test_codon_loglik_c3(precision, mode):
+    """BASELINE configs[3] (256-tip random tree, GY94+G4) at 2,000 patterns."""
+    w = config_workload("c3", seed=1, p=2_000)
+    tl = gpu_setup(w, mode, precision)
+    got = tl.loglik()
+    ora = oracle_run(w)
+    assert rel(got, ora.lnl) <= LNL_TOL[precision], (got, ora.lnl)
+    tl.close()
+
+
+@pytest.mark.parametrize("precision", [64, 32])
+@pytest.mark.parametrize("c,p", [(4, 130), (1, 64), (2, 65)])
+def test_codon_per_node_partials(precision, c, p):
+    w = make_workload(tree_kind="yule", n=24, p=p, model="gy94", c=c, seed=5, missing_frac=0.05)
+    tl = gpu_setup(w, "reroot", precision)
+    tl.update()
+    ora = oracle_run(w, tree=rooted(tl), keep_partials=True)
+    worst = 0.0
+    for v, L in ora.partials.items():
+        err = node_partial_error(tl.partials(v), tl.scale(v - w.n), L, ora.cum_exponent[v])
+        worst = max(worst, float(err.max()))
+    assert worst <= NODE_TOL[precision], worst
+    assert rel(tl.root_loglik(), ora.lnl) <= LNL_TOL[precision]
+    tl.close()
+
+
+def test_codon_edge_pulley():
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="balanced", n=8, p=100, model="gy94", c=4, seed=12)
+    tl = gpu_setup(w, "level", 64)
+    root_l = tl.loglik()
+    t = w.tree
+    a, b = pruning.children_of(t.parent)[t.root]
     R.rrl_update_transition_matrices(tl.inst, 0, np.array([a], np.int32),
                                      np.array([t.blen[a] + t.blen[b]]))
     e = R.rrl_calculate_edge_log_likelihoods(tl.inst, b, a, a, 0, 0, b - w.n, a - w.n)
