@@ -43,6 +43,7 @@ CONFIG_DESC = {
     "c1": "configs[1]: 128-tip pectinate rerooted vs original, GTR+G4, 10,000 patterns per GPU",
     "c2": "configs[2]: 1,024-tip Yule rerooted, GTR+G4, 100,000 patterns per GPU",
     "c2_paper": "1,024-tip paper-random (PAPER.md:148) rerooted, GTR+G4, 100,000 patterns per GPU",
+    "c3": "configs[3]: 256-tip paper-random rerooted, GY94+G4 (61 states), 10,000 patterns per GPU",
     "c4": "configs[4]: 4,096-tip pectinate rerooted, GTR+G4, 4,194,304 patterns (strong scaling)",
 }
 METRIC = "updatePartials GFLOPS rerooted vs original root; %HBM roofline; 1/2/4/8 GPU"
@@ -137,7 +138,8 @@ def rank_workload(cfg: str, rank: int, world: int, seed: int = 1):
 
 
 def ncu_traffic(cfg: str, precision: int):
-    """DRAM bytes per updatePartials launch from the committed ncu capture."""
+    """DRAM bytes per updatePartials launch from the committed ncu capture
+    (profiles/ncu_traffic.json); null when there is none for this config."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         d = json.load(open(path))
@@ -360,12 +362,23 @@ def main():
                          "kernel": "k_partials_nuc / k_partials_nuc_bulk (updatePartials, one "
                                    "launch per level set)",
                          "algorithmic_bytes_per_pass": bpp,
+                         "algorithmic_bytes_per_launch": bpp / max(1.0, prof["partials_launches"] / nsi),
                          "launches_per_pass": prof["partials_launches"] / nsi,
                          "peak_source": f"{peak_src} hbm_gbs (MEASURED_PEAKS.json)",
                          "timing": "per-launch CUDA events on the launching stream, eager "
                                    f"instrumented pass of {nsi} steps after the timed region"},
             "lnL": float(d_out.item()),
         }
+        if s == 61:
+            # SIMT codon kernel: bound by FP32/FP64 FMA issue, not HBM
+            peak_tf = 148 * 128 * 2 * 1.965e9 / 1e12 if precision == 32 else 148 * 64 * 2 * 1.965e9 / 1e12
+            ach = fl / (part_ms * 1e-3) / 1e12
+            res["roofline"].update({
+                "bound": "alu", "achieved": ach, "peak": peak_tf, "unit": "TFLOP/s",
+                "frac": ach / peak_tf, "hbm_achieved_gbs": achieved,
+                "peak_source": "derived: 148 SMs x 128 FP32 (64 FP64) lanes x 2 flop x 1.965 GHz "
+                               "(B200_PROFILING.md clocks; DESIGN.md §6)",
+                "flops": "effective Eq.(1) flops (n-1) c s (4s-1) per pattern (reading A16)"})
         if with_original and cfg != "c4":
             to = make(w, "level", precision, False)
             ms_o, _ = timed(to, steps, warmup)
