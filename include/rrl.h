@@ -78,6 +78,8 @@ extern "C" {
 #define RRL_FLAG_CUDA_GRAPH 0x2u       /* capture each distinct operation list's
                                           level-set launches in a CUDA graph and
                                           replay it on later identical calls */
+#define RRL_FLAG_CODON_SIMT 0x4u       /* 61-state fp32: use the FP32 SIMT kernel
+                                          instead of the tcgen05 (3xTF32) one */
 
 /* Schedule flags (rrl_reroot_and_schedule). Low byte = mode. */
 #define RRL_SCHED_SEQUENTIAL 1u  /* post-order, one op per set (Fig.2 upper) */
@@ -106,8 +108,10 @@ typedef struct rrl_op {
   int32_t matrix2;
 } rrl_op;
 
-/* Kernel timing collected when profiling is enabled (CUDA events on the
- * instance stream around every launch; adds a small gap per launch). */
+/* Kernel timing collected when profiling is enabled: CUDA events on the
+ * instance stream around every eager launch, or around each CUDA-graph replay
+ * of a whole updatePartials call (RRL_FLAG_CUDA_GRAPH), whose time is then
+ * attributed to its partials_launches. */
 typedef struct rrl_profile {
   double partials_ms;          /* sum of updatePartials set-launch durations */
   int64_t partials_launches;   /* number of updatePartials launches */

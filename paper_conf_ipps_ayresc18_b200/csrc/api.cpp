@@ -78,10 +78,6 @@ struct Instance {
   std::vector<int32_t> last_offs;
   bool ops_valid = false;
   cudaGraphExec_t graph = nullptr;       // replay of the set launches
-  cudaGraphExec_t graph_prof = nullptr;  // same, with an external event between sets
-  std::vector<cudaEvent_t> gev;          // events of graph_prof (nsets + 1)
-  bool gev_pending = false;
-  int gev_nsets = 0;
   cudaStream_t graph_stream = nullptr;
   int graph_kernels = 0;
 
@@ -178,26 +174,9 @@ void drain_events(Instance *I) {
   I->events.clear();
 }
 
-// Sum the per-set durations of the last profiled graph replay.
-int drain_graph_events(Instance *I) {
-  if (!I->gev_pending) return 0;
-  CK(cudaEventSynchronize(I->gev[I->gev_nsets]));
-  for (int k = 0; k < I->gev_nsets; ++k) {
-    float ms = 0.f;
-    CK(cudaEventElapsedTime(&ms, I->gev[k], I->gev[k + 1]));
-    I->prof.partials_ms += ms;
-  }
-  I->gev_pending = false;
-  return 0;
-}
-
 int drop_graphs(Instance *I) {
-  int r = drain_graph_events(I);
-  if (r < 0) return r;
   if (I->graph) cudaGraphExecDestroy(I->graph);
-  if (I->graph_prof) cudaGraphExecDestroy(I->graph_prof);
   I->graph = nullptr;
-  I->graph_prof = nullptr;
   return 0;
 }
 
@@ -205,8 +184,6 @@ void destroy(Instance *I) {
   cudaSetDevice(I->device);
   if (I->stream) cudaStreamSynchronize(I->stream);
   if (I->graph) cudaGraphExecDestroy(I->graph);
-  if (I->graph_prof) cudaGraphExecDestroy(I->graph_prof);
-  for (auto e : I->gev) cudaEventDestroy(e);
   for (void *t : I->tip_partials)
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
@@ -712,23 +689,21 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
     if (rg < 0) return rg;
   }
 
-  // events_in_graph: record an external event before every set launch and
-  // after the last one (profiling inside a graph replay); otherwise, when
-  // profiling eagerly, bracket each launch with its own events.
-  auto launch_all = [&](bool capturing, bool events_in_graph) -> int {
+  auto launch_all = [&](bool capturing) -> int {
     for (int k = 0; k < nsets; ++k) {
       const int n = offs[k + 1] - offs[k];
-      if (events_in_graph) CK(cudaEventRecordWithFlags(I->gev[k], I->stream, cudaEventRecordExternal));
-      Timed tm(I, 0, !capturing);
+      Timed tm(I, 0, !capturing);  // eager profiling: one event pair per set launch
       int e = (I->s == 4) ? launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k],
                                                        I->h_ops + offs[k], n, I->p, I->p_pad, I->stream)
-                          : launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k],
-                                                         I->h_ops + offs[k], n, I->p, I->p_pad, I->stream);
+                          : (I->prec == 32 && I->c <= 4 && !(I->flags & RRL_FLAG_CODON_SIMT))
+                                ? launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, I->p, I->p_pad,
+                                                                  I->stream)
+                                : launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k],
+                                                               I->h_ops + offs[k], n, I->p, I->p_pad, I->stream);
       if (e == (int)cudaErrorNotSupported) return fail(RRL_ERROR_NO_IMPLEMENTATION, "kernel variant");
       if (e != 0) return fail(RRL_ERROR_CUDA, std::string("updatePartials launch: ") +
                                                   cudaGetErrorString(static_cast<cudaError_t>(e)));
     }
-    if (events_in_graph) CK(cudaEventRecordWithFlags(I->gev[nsets], I->stream, cudaEventRecordExternal));
     return 0;
   };
   int kl = 0;
@@ -737,42 +712,33 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
   // (the legacy default stream cannot be captured: eager launches there)
   const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && I->stream != nullptr;
   if (use_graph) {
-    const bool prof = I->profiling;
-    cudaGraphExec_t &gx = prof ? I->graph_prof : I->graph;
-    if ((I->graph || I->graph_prof) && I->graph_stream != I->stream) {
+    if (I->graph && I->graph_stream != I->stream) {
       int r = drop_graphs(I);
       if (r < 0) return r;
     }
-    if (prof) {
-      int r = drain_graph_events(I);
-      if (r < 0) return r;
-      while ((int)I->gev.size() < nsets + 1) {
-        cudaEvent_t e;
-        CK(cudaEventCreate(&e));
-        I->gev.push_back(e);
-      }
-    }
-    if (!gx) {
+    if (!I->graph) {
       cudaGraph_t g;
       CK(cudaStreamBeginCapture(I->stream, cudaStreamCaptureModeThreadLocal));
-      int e = launch_all(true, prof);
+      int e = launch_all(true);
       cudaError_t ce = cudaStreamEndCapture(I->stream, &g);
       if (e < 0) return e;
       CK(ce);
-      cudaError_t ie = cudaGraphInstantiate(&gx, g, 0);
+      cudaError_t ie = cudaGraphInstantiate(&I->graph, g, 0);
       cudaGraphDestroy(g);
       CK(ie);
       I->graph_stream = I->stream;
       I->graph_kernels = kl;
     }
-    CK(cudaGraphLaunch(gx, I->stream));
-    if (prof) {
-      I->gev_pending = true;
-      I->gev_nsets = nsets;
+    {
+      // profiling: one event pair around the whole replay on the launching
+      // stream; per-launch duration = region time / launches (events inside
+      // the graph would break the programmatic-dependent-launch overlap).
+      Timed tm(I, 0);
+      CK(cudaGraphLaunch(I->graph, I->stream));
     }
     I->prof.graph_launches += 1;
   } else {
-    int e = launch_all(false, false);
+    int e = launch_all(false);
     if (e < 0) return e;
   }
   I->prof.kernel_launches += kl;
@@ -921,8 +887,6 @@ int rrl_get_profile(int inst, rrl_profile *out) {
   if (!out) return fail(RRL_ERROR_GENERAL, "out NULL");
   CK(cudaStreamSynchronize(I->stream));
   drain_events(I);
-  int r = drain_graph_events(I);
-  if (r < 0) return r;
   *out = I->prof;
   return RRL_SUCCESS;
 }
@@ -931,8 +895,6 @@ int rrl_reset_profile(int inst) {
   GET(I, inst);
   CK(cudaStreamSynchronize(I->stream));
   drain_events(I);
-  int r = drain_graph_events(I);
-  if (r < 0) return r;
   I->prof = rrl_profile{};
   return RRL_SUCCESS;
 }

@@ -289,22 +289,23 @@ def test_codon_transition_matrices(precision):
     tl.close()
 
 
-@pytest.mark.parametrize("precision", [64, 32])
+@pytest.mark.parametrize("precision,simt", [(64, True), (32, True), (32, False)])
 @pytest.mark.parametrize("mode", ["reroot", "level"])
-def test_codon_loglik_c3(precision, mode):
-    """BASELINE configs[3] (256-tip random tree, GY94+G4) at 2,000 patterns."""
+def test_codon_loglik_c3(precision, simt, mode):
+    """BASELINE configs[3] (256-tip random tree, GY94+G4) at 2,000 patterns;
+    fp32 on both the SIMT kernel and the tcgen05 3xTF32 kernel."""
     w = config_workload("c3", seed=1, p=2_000)
-    tl = gpu_setup(w, mode, precision)
+    tl = gpu_setup(w, mode, precision, codon_simt=simt)
     got = tl.loglik()
     ora = oracle_run(w)
     assert rel(got, ora.lnl) <= LNL_TOL[precision], (got, ora.lnl)
     tl.close()
 
 
-@pytest.mark.parametrize("precision", [64, 32])
-@pytest.mark.parametrize("c,p", [(4, 130), (1, 64), (2, 65)])
+@pytest.mark.parametrize("precision,simt", [(64, True), (32, True), (32, False)])
+@pytest.mark.parametrize("c,p", [(4, 130), (1, 64), (2, 65), (4, 1000), (8, 300)])
 @pytest.mark.parametrize("matrices", ["oracle_expm", "gpu_k1"])
-def test_codon_per_node_partials(precision, c, p, matrices):
+def test_codon_per_node_partials(precision, simt, c, p, matrices):
     """Per-node codon partials.  With the oracle's own expm matrices loaded
     through rrl_set_transition_matrix the K3 arithmetic is checked at the
     fp64 node tolerance.  With the GPU's eigen-route K1 matrices, codon P has
@@ -313,7 +314,7 @@ def test_codon_per_node_partials(precision, c, p, matrices):
     (reading "codon node tolerance"), so fp64 is held to 1e-6 there."""
     from paper_conf_ipps_ayresc18_b200 import rrl as R
     w = make_workload(tree_kind="yule", n=24, p=p, model="gy94", c=c, seed=5, missing_frac=0.05)
-    tl = gpu_setup(w, "reroot", precision)
+    tl = gpu_setup(w, "reroot", precision, codon_simt=simt)
     rt = rooted(tl)
     if matrices == "gpu_k1":
         tl.update()
