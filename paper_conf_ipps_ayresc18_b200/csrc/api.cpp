@@ -695,7 +695,7 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
       Timed tm(I, 0, !capturing);  // eager profiling: one event pair per set launch
       int e = (I->s == 4) ? launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k],
                                                        I->h_ops + offs[k], n, I->p, I->p_pad, I->stream)
-                          : (I->prec == 32 && I->c <= 4 && !(I->flags & RRL_FLAG_CODON_SIMT))
+                          : (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))
                                 ? launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, I->p, I->p_pad,
                                                                   I->stream)
                                 : launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k],

@@ -8,22 +8,28 @@
 // This is the one place on the hot path that really is a dense contraction
 // (BASELINE north star), so it runs on tcgen05:
 //  * M = 128 patterns (TMEM lanes), N = 64 states (61 padded), K = 64 child
-//    states in 8 steps of K = 8 (tf32).  The 2 children x C categories
-//    accumulators use all 512 TMEM columns for C = 4.
+//    states in 8 steps of K = 8 (tf32).
 //  * fp32 accuracy with 3xTF32: x = hi + lo with hi = x with the low 13
-//    mantissa bits cleared (exact) and lo = x - hi (exact); the tensor core
-//    reads the top 19 bits of each operand, so hi*hi + hi*lo + lo*hi carries
-//    ~2^-22 relative error per product, fp32 accumulation.  A tip child's A
-//    tile is one-hot (or all ones for a missing state -> row sums), exact in
-//    tf32, so only hi*hi + hi*lo is issued for it.
+//    mantissa bits cleared (exact) and lo = x - hi (exact).  hi*hi goes to a
+//    main accumulator, hi*lo + lo*hi to a separate correction accumulator: the
+//    MMA aligns every addend to its accumulator's magnitude with ~20 bits, so
+//    corrections ~2^-11 smaller than the main terms would lose most of their
+//    bits in a shared accumulator (measured: 4e-6 vs 9e-7 per product with
+//    tools/diag_codon_tc.py).  A tip child's A tile is one-hot (or all ones
+//    for a missing state -> row sums), exact in tf32, so its lo*hi is skipped.
+//  * TMEM: two category buffers x 2 children x (main, correction) x 64
+//    columns = 512 columns, so category c+1's MMAs never wait for category
+//    c's epilogue to drain TMEM.
 //  * Operands are built by all 256 threads straight into the canonical
 //    no-swizzle K-major UMMA layout (8-row x 16-byte core matrices; LBO = 128 B
 //    between the two K halves, SBO = 256 B between 8-row groups), published to
 //    the async proxy (fence.proxy.async), and one elected thread issues the
 //    MMAs and tcgen05.commit's them to an mbarrier.
-//  * Epilogue: warps 0-3 own TMEM lane quarters (one pattern per thread);
-//    pass 1 takes max over (c, z) of D_1 .* D_2 (tcgen05.ld 32x32b.x16), pass
-//    2 scales by the exact 2^-e and stores rows of 64 states.
+//  * Epilogue per category: warps 0-3 own TMEM lane quarters (one pattern per
+//    thread; tcgen05.ld 32x32b.x16): (main1 + corr1) * (main2 + corr2) is
+//    stored unscaled while the running max over (c, z) is kept; once all
+//    categories are done the thread rescales its own rows by the exact 2^-e
+//    (an L2-resident re-read of 256 B per category).
 // Persistent CTAs (one per SM: the CTA owns all of TMEM) walk the flattened
 // (operation, tile) space of the level set.
 #include <cuda_runtime.h>
@@ -144,6 +150,11 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
   asm volatile("griddepcontrol.launch_dependents;" :::);
 
   uint32_t phase = 0;
+  // TMEM columns: two category buffers of 256 columns; per buffer and child b
+  // the main accumulator (hi*hi) at 128 b and the correction accumulator
+  // (hi*lo + lo*hi) at 128 b + 64.  Keeping the ~2^-11-smaller corrections in
+  // their own accumulator keeps them accurate (the MMA aligns every addend to
+  // the accumulator's magnitude with ~20 bits); they meet in fp32 in the epilogue.
   for (int f = blockIdx.x; f < total; f += gridDim.x) {
     const DevOp &op = ops[f / ntiles];
     const int p0 = (f % ntiles) * TM;
@@ -155,40 +166,74 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
         const int pp = p0 + tid;
         st_s[b * TM + tid] = pp < p ? static_cast<const uint8_t *>(in[b])[pp] : (uint8_t)kS61;
       }
+    const int r = warp * 32 + lane;  // epilogue row (warps 0-3)
+    const int pp = p0 + r;
+    const bool valid = warp < 4 && pp < p;
+    float *out = static_cast<float *>(op.out);
+    const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16);
+    float m = 0.f;
+
+    // product of category cc from TMEM buffer cc&1 -> out (unscaled), running max
+    auto epilogue_cat = [&](int cc) {
+      const uint32_t cb = lane_base + (uint32_t)((cc & 1) * 256);
+#pragma unroll
+      for (int q = 0; q < TS / 16; ++q) {
+        float m1[16], c1[16], m2[16], c2[16];
+        tmem_ld16(cb + 0 + q * 16, m1);
+        tmem_ld16(cb + 64 + q * 16, c1);
+        tmem_ld16(cb + 128 + q * 16, m2);
+        tmem_ld16(cb + 192 + q * 16, c2);
+        tmem_wait_ld();
+        float v[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          v[i] = (m1[i] + c1[i]) * (m2[i] + c2[i]);
+          m = fmaxf(m, v[i]);
+        }
+        if (valid) {
+          float4 *dst = reinterpret_cast<float4 *>(out + ((size_t)cc * p_pad + pp) * TS + q * 16);
+#pragma unroll
+          for (int i = 0; i < 4; ++i) dst[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
+        }
+      }
+    };
 
     for (int c = 0; c < C; ++c) {
-      if (c > 0) {  // MMAs of category c-1 must be done reading the operand tiles
+      if (c > 0) {  // MMAs of category c-1 done: operand smem free, its products ready
         bar_wait(bar, phase);
         phase ^= 1u;
+        fence_after();
+        if (warp < 4) epilogue_cat(c - 1);
+        fence_before();
       }
-      __syncthreads();  // tip states visible; previous tile's epilogue done
+      __syncthreads();  // tip states visible; smem and TMEM buffer c&1 free
       // ---- operand tiles for category c (both children), hi/lo split
       for (int b = 0; b < 2; ++b) {
         const uint32_t a_hi = sbase + SMEM_A + (2 * b) * A_BYTES, a_lo = a_hi + A_BYTES;
         if (!tip[b]) {
           const float *A = static_cast<const float *>(in[b]) + ((size_t)c * p_pad + p0) * TS;
           for (int i = tid; i < TM * 16; i += kThr) {
-            const int kh = i & 1, r = (i >> 1) & (TM - 1), kb = i >> 8;
+            const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
             const int j = kb * 2 + kh;
             float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (p0 + r < p) v = __ldg(reinterpret_cast<const float4 *>(A + (size_t)r * TS + j * 4));
-            const uint32_t o = umma_off(r, j, TM);
+            if (p0 + rr < p) v = __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + j * 4));
+            const uint32_t o = umma_off(rr, j, TM);
             const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
             sts128(a_hi + o, h0, h1, h2, h3);
             sts128(a_lo + o, v.x - h0, v.y - h1, v.z - h2, v.w - h3);
           }
         } else {
           for (int i = tid; i < TM * 16; i += kThr) {
-            const int kh = i & 1, r = (i >> 1) & (TM - 1), kb = i >> 8;
+            const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
             const int j = kb * 2 + kh;
-            const unsigned s = st_s[b * TM + r];
+            const unsigned sv = st_s[b * TM + rr];
             float v[4];
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
               const unsigned k = (unsigned)(j * 4 + q);
-              v[q] = (s < (unsigned)kS61) ? (k == s ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
+              v[q] = (sv < (unsigned)kS61) ? (k == sv ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
             }
-            sts128(a_hi + umma_off(r, j, TM), v[0], v[1], v[2], v[3]);
+            sts128(a_hi + umma_off(rr, j, TM), v[0], v[1], v[2], v[3]);
           }
         }
         const uint32_t b_hi = sbase + SMEM_B + (2 * b) * B_BYTES, b_lo = b_hi + B_BYTES;
@@ -209,16 +254,16 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       if (tid == 0) {
         fence_after();
         for (int b = 0; b < 2; ++b) {
-          const uint32_t d = tmem + (uint32_t)((2 * c + b) * TS);
+          const uint32_t dm = tmem + (uint32_t)((c & 1) * 256 + b * 128), dc = dm + 64;
           const uint32_t a_hi = sbase + SMEM_A + (2 * b) * A_BYTES, a_lo = a_hi + A_BYTES;
           const uint32_t b_hi = sbase + SMEM_B + (2 * b) * B_BYTES, b_lo = b_hi + B_BYTES;
 #pragma unroll
           for (int kb = 0; kb < TS / 8; ++kb) {
             const uint64_t ah = umma_desc(a_hi + kb * (TM * 32)), al = umma_desc(a_lo + kb * (TM * 32));
             const uint64_t bh = umma_desc(b_hi + kb * (TS * 32)), bl = umma_desc(b_lo + kb * (TS * 32));
-            mma_tf32(d, ah, bh, kb > 0 ? 1u : 0u);
-            mma_tf32(d, ah, bl, 1u);
-            if (!tip[b]) mma_tf32(d, al, bh, 1u);
+            mma_tf32(dm, ah, bh, kb > 0 ? 1u : 0u);
+            mma_tf32(dc, ah, bl, kb > 0 ? 1u : 0u);
+            if (!tip[b]) mma_tf32(dc, al, bh, 1u);
           }
         }
         mma_commit(bar);
@@ -227,26 +272,9 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
     bar_wait(bar, phase);  // last category's products are in TMEM
     phase ^= 1u;
     fence_after();
-
-    // ---- epilogue: warps 0-3, one pattern (TMEM lane) per thread
     if (warp < 4) {
-      const int r = warp * 32 + lane;
-      const int pp = p0 + r;
-      const bool valid = pp < p;
-      const uint32_t lane_base = tmem + ((uint32_t)(warp * 32) << 16);
-      float m = 0.f;
-      if (op.scale_out != nullptr) {
-        for (int c = 0; c < C; ++c)
-#pragma unroll
-          for (int q = 0; q < TS / 16; ++q) {
-            float a[16], bb[16];
-            tmem_ld16(lane_base + (uint32_t)((2 * c) * TS + q * 16), a);
-            tmem_ld16(lane_base + (uint32_t)((2 * c + 1) * TS + q * 16), bb);
-            tmem_wait_ld();
-#pragma unroll
-            for (int i = 0; i < 16; ++i) m = fmaxf(m, a[i] * bb[i]);
-          }
-      }
+      epilogue_cat(C - 1);
+      // ---- rescale: e from max over (c, z); rows re-read by the thread that wrote them
       int e = 0;
       if (op.scale_out != nullptr) {
         e = frexp_e(m);
@@ -259,23 +287,18 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       } else if (op.scale_in != nullptr) {
         e = valid ? op.scale_in[pp] : 0;
       }
-      const float sc = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
-      float *out = static_cast<float *>(op.out);
-      for (int c = 0; c < C; ++c)
-#pragma unroll
-        for (int q = 0; q < TS / 16; ++q) {
-          float a[16], bb[16];
-          tmem_ld16(lane_base + (uint32_t)((2 * c) * TS + q * 16), a);
-          tmem_ld16(lane_base + (uint32_t)((2 * c + 1) * TS + q * 16), bb);
-          tmem_wait_ld();
-          if (valid) {
-            float4 *dst = reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + pp) * TS + q * 16);
-#pragma unroll
-            for (int i = 0; i < 4; ++i)
-              dst[i] = make_float4(a[4 * i] * bb[4 * i] * sc, a[4 * i + 1] * bb[4 * i + 1] * sc,
-                                   a[4 * i + 2] * bb[4 * i + 2] * sc, a[4 * i + 3] * bb[4 * i + 3] * sc);
+      if (valid && e != 0) {
+        const float sc = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
+        for (int c = 0; c < C; ++c) {
+          float4 *row = reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + pp) * TS);
+#pragma unroll 4
+          for (int i = 0; i < TS / 4; ++i) {
+            float4 v = row[i];
+            v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
+            row[i] = v;
           }
         }
+      }
     }
     fence_before();
     __syncthreads();  // TMEM and tip-state smem free for the next tile
@@ -315,15 +338,15 @@ int launch_tc(const DevOp *d_ops, int nops, int p, int p_pad, cudaStream_t st) {
 
 }  // namespace
 
-// fp32 codon instances with c <= 4 (the accumulators of 2 children x c
-// categories x 64 columns fit the 512 TMEM columns); returns
-// cudaErrorNotSupported otherwise so the caller uses the SIMT kernel.
+// fp32 codon instances, c in {1, 2, 4, 8}; cudaErrorNotSupported otherwise
+// (the caller then uses the SIMT kernel).
 int launch_update_partials_codon_tc(int c, const DevOp *d_ops, int nops, int p, int p_pad, void *stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   switch (c) {
     case 1: return launch_tc<1>(d_ops, nops, p, p_pad, st);
     case 2: return launch_tc<2>(d_ops, nops, p, p_pad, st);
     case 4: return launch_tc<4>(d_ops, nops, p, p_pad, st);
+    case 8: return launch_tc<8>(d_ops, nops, p, p_pad, st);
     default: return (int)cudaErrorNotSupported;
   }
 }
