@@ -9,29 +9,30 @@
 // (BASELINE north star), so it runs on tcgen05:
 //  * M = 128 patterns (TMEM lanes), N = 64 states (61 padded), K = 64 child
 //    states in 8 steps of K = 8 (tf32).
-//  * fp32 accuracy with 3xTF32: x = hi + lo with hi = x with the low 13
-//    mantissa bits cleared (exact) and lo = x - hi (exact).  hi*hi goes to a
-//    main accumulator, hi*lo + lo*hi to a separate correction accumulator: the
-//    MMA aligns every addend to its accumulator's magnitude with ~20 bits, so
-//    corrections ~2^-11 smaller than the main terms would lose most of their
-//    bits in a shared accumulator (measured: 4e-6 vs 9e-7 per product with
-//    tools/diag_codon_tc.py).  A tip child's A tile is one-hot (or all ones
-//    for a missing state -> row sums), exact in tf32, so its lo*hi is skipped.
-//  * TMEM: two category buffers x 2 children x (main, correction) x 64
-//    columns = 512 columns, so category c+1's MMAs never wait for category
-//    c's epilogue to drain TMEM.
-//  * Operands are built by all 256 threads straight into the canonical
-//    no-swizzle K-major UMMA layout (8-row x 16-byte core matrices; LBO = 128 B
-//    between the two K halves, SBO = 256 B between 8-row groups), published to
-//    the async proxy (fence.proxy.async), and one elected thread issues the
-//    MMAs and tcgen05.commit's them to an mbarrier.
-//  * Epilogue per category: warps 0-3 own TMEM lane quarters (one pattern per
-//    thread; tcgen05.ld 32x32b.x16): (main1 + corr1) * (main2 + corr2) is
-//    stored unscaled while the running max over (c, z) is kept; once all
-//    categories are done the thread rescales its own rows by the exact 2^-e
-//    (an L2-resident re-read of 256 B per category).
-// Persistent CTAs (one per SM: the CTA owns all of TMEM) walk the flattened
-// (operation, tile) space of the level set.
+//  * fp32 accuracy with 3xTF32: x = hi + lo, hi = x with the low 13 mantissa
+//    bits cleared (exact), lo = x - hi (exact).  The MMA aligns the addends of
+//    an accumulation to the accumulator with ~20 bits and truncates, which
+//    costs ~0.5 ulp of bias per accumulation step (tools/diag_codon_tc.py:
+//    9e-7 for a 64-term sum in one accumulator vs 6e-7 on SIMT FP32).  So the
+//    hi*hi terms go to four accumulators (two K steps each) and the
+//    ~2^-11-smaller hi*lo + lo*hi corrections to a fifth; the five meet in
+//    fp32 in the epilogue.  A tip child's A tile is one-hot (all ones for a
+//    missing state -> row sums), exact in tf32, so its lo*hi is skipped.
+//  * Work is a pipeline of phases (tile, category, child): while the MMAs of
+//    phase k run, all 256 threads build phase k+1's operands (global loads,
+//    hi/lo split) into the other half of a double-buffered shared-memory ring,
+//    directly in the canonical no-swizzle K-major UMMA layout (8-row x 16-byte
+//    core matrices; LBO = 128 B between the two K halves, SBO = 256 B between
+//    8-row groups), published to the async proxy with fence.proxy.async; one
+//    thread issues the MMAs and tcgen05.commit's them to an mbarrier.
+//  * Epilogue of a phase: all 8 warps (warp w: TMEM lane quarter w%4, column
+//    half w/4) sum the five accumulators (tcgen05.ld 32x32b.x16).  Child 1's
+//    result is parked in shared memory; child 2's is multiplied with it,
+//    stored unscaled and folded into the running max over (c, z).  After the
+//    last category the two column halves exchange their maxima, and every
+//    thread rescales its own rows by the exact 2^-e (an L2-resident re-read).
+// Persistent CTAs (one per SM: 320 TMEM columns, ~225 KB of shared memory)
+// walk the flattened (operation, tile) space of the level set.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -47,13 +48,18 @@ constexpr int kS61 = 61;
 constexpr int kThr = 256;
 constexpr int A_BYTES = TM * TS * 4;  // 32 KB per operand tile
 constexpr int B_BYTES = TS * TS * 4;  // 16 KB
-// smem: A[child][hi,lo], B[child][hi,lo]
-constexpr int SMEM_A = 0;
-constexpr int SMEM_B = 4 * A_BYTES;
-constexpr int SMEM_ST = SMEM_B + 4 * B_BYTES;   // tip states [2][128]
-constexpr int SMEM_BAR = SMEM_ST + 2 * TM;      // mbarrier
-constexpr int SMEM_TMEM = SMEM_BAR + 8;         // TMEM base address
+constexpr int BUF_BYTES = 2 * A_BYTES + 2 * B_BYTES;  // A hi/lo + B hi/lo of one phase
+constexpr int S1_STRIDE = TS + 1;
+// smem: 2 operand buffers, child-1 result, tip states [tile parity][child][128],
+// row maxima [2 halves][128], mbarrier, TMEM base address
+constexpr int SMEM_BUF = 0;
+constexpr int SMEM_S1 = 2 * BUF_BYTES;
+constexpr int SMEM_ST = SMEM_S1 + TM * S1_STRIDE * 4;
+constexpr int SMEM_MX = SMEM_ST + 2 * 2 * TM;
+constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;
+constexpr int SMEM_TMEM = SMEM_BAR + 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 8;
+constexpr int kTmemCols = 512;  // 5 x 64 used (4 main + 1 correction accumulators)
 
 __device__ inline uint32_t smem_addr(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -128,13 +134,15 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(sm + SMEM_TMEM);
   uint8_t *st_s = sm + SMEM_ST;
+  float *S1 = reinterpret_cast<float *>(sm + SMEM_S1);
+  float *mx = reinterpret_cast<float *>(sm + SMEM_MX);
   const uint32_t sbase = smem_addr(sm);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
   if (warp == 0) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                      smem_addr(tmem_slot)),
-                 "r"(512));
+                 "r"(kTmemCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   if (tid == 0) {
@@ -149,163 +157,195 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" :::);
 
-  uint32_t phase = 0;
-  // TMEM columns: two category buffers of 256 columns; per buffer and child b
-  // the main accumulator (hi*hi) at 128 b and the correction accumulator
-  // (hi*lo + lo*hi) at 128 b + 64.  Keeping the ~2^-11-smaller corrections in
-  // their own accumulator keeps them accurate (the MMA aligns every addend to
-  // the accumulator's magnitude with ~20 bits); they meet in fp32 in the epilogue.
-  for (int f = blockIdx.x; f < total; f += gridDim.x) {
+  const int my_tiles = total > (int)blockIdx.x ? (total - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+  const int nphase = my_tiles * C * 2;  // phases (tile, category, child)
+
+  // tip states of local tile lt (parity lt & 1)
+  auto load_states = [&](int lt) {
+    const int f = blockIdx.x + lt * gridDim.x;
     const DevOp &op = ops[f / ntiles];
     const int p0 = (f % ntiles) * TM;
-    const bool tip[2] = {(op.flags & OP_TIP1) != 0, (op.flags & OP_TIP2) != 0};
     const void *in[2] = {op.in1, op.in2};
-    const float *Pg[2] = {static_cast<const float *>(op.P1), static_cast<const float *>(op.P2)};
+    const int fl[2] = {op.flags & OP_TIP1, op.flags & OP_TIP2};
     for (int b = 0; b < 2; ++b)
-      if (tip[b] && tid < TM) {
+      if (fl[b] && tid < TM) {
         const int pp = p0 + tid;
-        st_s[b * TM + tid] = pp < p ? static_cast<const uint8_t *>(in[b])[pp] : (uint8_t)kS61;
+        st_s[((lt & 1) * 2 + b) * TM + tid] = pp < p ? static_cast<const uint8_t *>(in[b])[pp] : (uint8_t)kS61;
       }
-    const int r = warp * 32 + lane;  // epilogue row (warps 0-3)
-    const int pp = p0 + r;
-    const bool valid = warp < 4 && pp < p;
-    float *out = static_cast<float *>(op.out);
-    const uint32_t lane_base = tmem + ((uint32_t)((warp & 3) * 32) << 16);
-    float m = 0.f;
+  };
 
-    // product of category cc from TMEM buffer cc&1 -> out (unscaled), running max
-    auto epilogue_cat = [&](int cc) {
-      const uint32_t cb = lane_base + (uint32_t)((cc & 1) * 256);
-#pragma unroll
-      for (int q = 0; q < TS / 16; ++q) {
-        float m1[16], c1[16], m2[16], c2[16];
-        tmem_ld16(cb + 0 + q * 16, m1);
-        tmem_ld16(cb + 64 + q * 16, c1);
-        tmem_ld16(cb + 128 + q * 16, m2);
-        tmem_ld16(cb + 192 + q * 16, c2);
-        tmem_wait_ld();
-        float v[16];
-#pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          v[i] = (m1[i] + c1[i]) * (m2[i] + c2[i]);
-          m = fmaxf(m, v[i]);
-        }
-        if (valid) {
-          float4 *dst = reinterpret_cast<float4 *>(out + ((size_t)cc * p_pad + pp) * TS + q * 16);
-#pragma unroll
-          for (int i = 0; i < 4; ++i) dst[i] = make_float4(v[4 * i], v[4 * i + 1], v[4 * i + 2], v[4 * i + 3]);
-        }
+  // operands of phase g into buffer g & 1
+  auto build = [&](int g) {
+    const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
+    const int f = blockIdx.x + lt * gridDim.x;
+    const DevOp &op = ops[f / ntiles];
+    const int p0 = (f % ntiles) * TM;
+    const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+    const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
+    const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+    if (!tip) {
+      const float *A = static_cast<const float *>(b == 0 ? op.in1 : op.in2) + ((size_t)c * p_pad + p0) * TS;
+      for (int i = tid; i < TM * 16; i += kThr) {
+        const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
+        const int j = kb * 2 + kh;
+        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (p0 + rr < p) v = __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + j * 4));
+        const uint32_t o = umma_off(rr, j, TM);
+        const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
+        sts128(a_hi + o, h0, h1, h2, h3);
+        sts128(a_lo + o, v.x - h0, v.y - h1, v.z - h2, v.w - h3);
       }
-    };
-
-    for (int c = 0; c < C; ++c) {
-      if (c > 0) {  // MMAs of category c-1 done: operand smem free, its products ready
-        bar_wait(bar, phase);
-        phase ^= 1u;
-        fence_after();
-        if (warp < 4) epilogue_cat(c - 1);
-        fence_before();
-      }
-      __syncthreads();  // tip states visible; smem and TMEM buffer c&1 free
-      // ---- operand tiles for category c (both children), hi/lo split
-      for (int b = 0; b < 2; ++b) {
-        const uint32_t a_hi = sbase + SMEM_A + (2 * b) * A_BYTES, a_lo = a_hi + A_BYTES;
-        if (!tip[b]) {
-          const float *A = static_cast<const float *>(in[b]) + ((size_t)c * p_pad + p0) * TS;
-          for (int i = tid; i < TM * 16; i += kThr) {
-            const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-            const int j = kb * 2 + kh;
-            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (p0 + rr < p) v = __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + j * 4));
-            const uint32_t o = umma_off(rr, j, TM);
-            const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
-            sts128(a_hi + o, h0, h1, h2, h3);
-            sts128(a_lo + o, v.x - h0, v.y - h1, v.z - h2, v.w - h3);
-          }
-        } else {
-          for (int i = tid; i < TM * 16; i += kThr) {
-            const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-            const int j = kb * 2 + kh;
-            const unsigned sv = st_s[b * TM + rr];
-            float v[4];
+    } else {
+      const uint8_t *sts = st_s + ((lt & 1) * 2 + b) * TM;
+      for (int i = tid; i < TM * 16; i += kThr) {
+        const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
+        const int j = kb * 2 + kh;
+        const unsigned sv = sts[rr];
+        float v[4];
 #pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              const unsigned k = (unsigned)(j * 4 + q);
-              v[q] = (sv < (unsigned)kS61) ? (k == sv ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
-            }
-            sts128(a_hi + umma_off(rr, j, TM), v[0], v[1], v[2], v[3]);
-          }
+        for (int q = 0; q < 4; ++q) {
+          const unsigned k = (unsigned)(j * 4 + q);
+          v[q] = (sv < (unsigned)kS61) ? (k == sv ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
         }
-        const uint32_t b_hi = sbase + SMEM_B + (2 * b) * B_BYTES, b_lo = b_hi + B_BYTES;
-        const float *P = Pg[b] + (size_t)c * TS * TS;  // natural [z][x] = K-major B
-        for (int i = tid; i < TS * 16; i += kThr) {
-          const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
-          const int j = kb * 2 + kh;
-          const float4 v = __ldg(reinterpret_cast<const float4 *>(P + z * TS + j * 4));
-          const uint32_t o = umma_off(z, j, TS);
-          const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
-          sts128(b_hi + o, h0, h1, h2, h3);
-          sts128(b_lo + o, v.x - h0, v.y - h1, v.z - h2, v.w - h3);
-        }
-      }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
-      fence_before();
-      __syncthreads();
-      if (tid == 0) {
-        fence_after();
-        for (int b = 0; b < 2; ++b) {
-          const uint32_t dm = tmem + (uint32_t)((c & 1) * 256 + b * 128), dc = dm + 64;
-          const uint32_t a_hi = sbase + SMEM_A + (2 * b) * A_BYTES, a_lo = a_hi + A_BYTES;
-          const uint32_t b_hi = sbase + SMEM_B + (2 * b) * B_BYTES, b_lo = b_hi + B_BYTES;
-#pragma unroll
-          for (int kb = 0; kb < TS / 8; ++kb) {
-            const uint64_t ah = umma_desc(a_hi + kb * (TM * 32)), al = umma_desc(a_lo + kb * (TM * 32));
-            const uint64_t bh = umma_desc(b_hi + kb * (TS * 32)), bl = umma_desc(b_lo + kb * (TS * 32));
-            mma_tf32(dm, ah, bh, kb > 0 ? 1u : 0u);
-            mma_tf32(dc, ah, bl, kb > 0 ? 1u : 0u);
-            if (!tip[b]) mma_tf32(dc, al, bh, 1u);
-          }
-        }
-        mma_commit(bar);
+        sts128(a_hi + umma_off(rr, j, TM), v[0], v[1], v[2], v[3]);
       }
     }
-    bar_wait(bar, phase);  // last category's products are in TMEM
+    const float *P = static_cast<const float *>(b == 0 ? op.P1 : op.P2) + (size_t)c * TS * TS;
+    for (int i = tid; i < TS * 16; i += kThr) {  // natural [z][x] layout = K-major B
+      const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
+      const int j = kb * 2 + kh;
+      const float4 v = __ldg(reinterpret_cast<const float4 *>(P + z * TS + j * 4));
+      const uint32_t o = umma_off(z, j, TS);
+      const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
+      sts128(b_hi + o, h0, h1, h2, h3);
+      sts128(b_lo + o, v.x - h0, v.y - h1, v.z - h2, v.w - h3);
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
+  };
+
+  // single thread: the MMAs of phase g (operands in buffer g & 1)
+  auto issue = [&](int g) {
+    const int lt = g / (2 * C), b = g & 1;
+    const int f = blockIdx.x + lt * gridDim.x;
+    const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+    const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
+    const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+#pragma unroll
+    for (int kb = 0; kb < TS / 8; ++kb) {
+      const uint64_t ah = umma_desc(a_hi + kb * (TM * 32)), al = umma_desc(a_lo + kb * (TM * 32));
+      const uint64_t bh = umma_desc(b_hi + kb * (TS * 32)), bl = umma_desc(b_lo + kb * (TS * 32));
+      const uint32_t dmain = tmem + (uint32_t)((kb >> 1) * TS), dcorr = tmem + (uint32_t)(4 * TS);
+      mma_tf32(dmain, ah, bh, (kb & 1) ? 1u : 0u);
+      mma_tf32(dcorr, ah, bl, kb > 0 ? 1u : 0u);
+      if (!tip) mma_tf32(dcorr, al, bh, 1u);
+    }
+    mma_commit(bar);
+  };
+
+  const int q = warp & 3, h = warp >> 2;  // TMEM lane quarter, column half
+  const int r = q * 32 + lane;            // this thread's row (pattern) in the tile
+  const uint32_t tl = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(h * 32);
+  float m = 0.f;
+  uint32_t phase = 0;
+
+  if (nphase > 0) {
+    load_states(0);
+    __syncthreads();
+    build(0);
+    fence_before();
+    __syncthreads();
+    if (tid == 0) {
+      fence_after();
+      issue(0);
+    }
+  }
+  for (int g = 0; g < nphase; ++g) {
+    const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
+    if (g + 1 < nphase) {
+      if ((g + 1) % (2 * C) == 0) {  // next phase starts a new tile: its tip states
+        load_states(lt + 1);
+        __syncthreads();
+      }
+      build(g + 1);  // overlaps the MMAs of phase g
+    }
+    bar_wait(bar, phase);
     phase ^= 1u;
     fence_after();
-    if (warp < 4) {
-      epilogue_cat(C - 1);
-      // ---- rescale: e from max over (c, z); rows re-read by the thread that wrote them
-      int e = 0;
-      if (op.scale_out != nullptr) {
-        e = frexp_e(m);
-        if (valid) {
-          int tot = e;
-          if (op.cum1 != nullptr) tot += op.cum1[pp];
-          if (op.cum2 != nullptr) tot += op.cum2[pp];
-          op.scale_out[pp] = tot;
-        }
-      } else if (op.scale_in != nullptr) {
-        e = valid ? op.scale_in[pp] : 0;
+    // ---- epilogue of phase g
+    const int f = blockIdx.x + lt * gridDim.x;
+    const DevOp &op = ops[f / ntiles];
+    const int p0 = (f % ntiles) * TM;
+    const int pp = p0 + r;
+    const bool valid = pp < p;
+    float d[32];
+#pragma unroll
+    for (int half = 0; half < 2; ++half) {
+      float a0[16], a1[16], a2[16], a3[16], cc[16];
+      tmem_ld16(tl + 0 * TS + half * 16, a0);
+      tmem_ld16(tl + 1 * TS + half * 16, a1);
+      tmem_ld16(tl + 2 * TS + half * 16, a2);
+      tmem_ld16(tl + 3 * TS + half * 16, a3);
+      tmem_ld16(tl + 4 * TS + half * 16, cc);
+      tmem_wait_ld();
+#pragma unroll
+      for (int i = 0; i < 16; ++i) d[half * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
+    }
+    float *s1row = S1 + r * S1_STRIDE + h * 32;
+    if (b == 0) {
+#pragma unroll
+      for (int i = 0; i < 32; ++i) s1row[i] = d[i];
+    } else {
+      float *out = static_cast<float *>(op.out);
+#pragma unroll
+      for (int i = 0; i < 32; ++i) {
+        d[i] *= s1row[i];
+        m = fmaxf(m, d[i]);
       }
-      if (valid && e != 0) {
-        const float sc = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
-        for (int c = 0; c < C; ++c) {
-          float4 *row = reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + pp) * TS);
-#pragma unroll 4
-          for (int i = 0; i < TS / 4; ++i) {
-            float4 v = row[i];
-            v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
-            row[i] = v;
+      if (valid) {
+        float4 *dst = reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + pp) * TS + h * 32);
+#pragma unroll
+        for (int i = 0; i < 8; ++i) dst[i] = make_float4(d[4 * i], d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
+      }
+      if (c == C - 1) {  // ---- tile done: exponent from max over (c, z), rescale own rows
+        mx[h * TM + r] = m;
+        __syncthreads();
+        const float mm = fmaxf(mx[r], mx[TM + r]);
+        int e = 0;
+        if (op.scale_out != nullptr) {
+          e = frexp_e(mm);
+          if (valid && h == 0) {
+            int tot = e;
+            if (op.cum1 != nullptr) tot += op.cum1[pp];
+            if (op.cum2 != nullptr) tot += op.cum2[pp];
+            op.scale_out[pp] = tot;
+          }
+        } else if (op.scale_in != nullptr) {
+          e = valid ? op.scale_in[pp] : 0;
+        }
+        if (valid && e != 0) {
+          const float sc = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
+          for (int cat = 0; cat < C; ++cat) {
+            float4 *row = reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + pp) * TS + h * 32);
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+              float4 v = row[i];
+              v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
+              row[i] = v;
+            }
           }
         }
+        m = 0.f;
       }
     }
     fence_before();
-    __syncthreads();  // TMEM and tip-state smem free for the next tile
-    fence_after();
+    __syncthreads();  // TMEM accumulators read, S1 / maxima settled, phase g+1 operands visible
+    if (g + 1 < nphase && tid == 0) {
+      fence_after();
+      issue(g + 1);
+    }
   }
   __syncthreads();
-  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(512));
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
 }
 
 template <int C>
