@@ -10,7 +10,9 @@
 //  * M = 128 patterns (TMEM lanes), N = 64 states (61 padded), K = 64 child
 //    states in 8 steps of K = 8 (tf32).
 //  * fp32 accuracy with 3xTF32: x = hi + lo, hi = x with the low 13 mantissa
-//    bits cleared (exact), lo = x - hi (exact).  The MMA aligns the addends of
+//    bits cleared (exact), lo = x - hi rounded to the nearest tf32 (the tensor
+//    core truncates operands to tf32; truncating lo would bias every
+//    correction by up to 2^-22 in one direction).  The MMA aligns the addends of
 //    an accumulation to the accumulator with ~20 bits and truncates, which
 //    costs ~0.5 ulp of bias per accumulation step (tools/diag_codon_tc.py:
 //    9e-7 for a 64-term sum in one accumulator vs 6e-7 on SIMT FP32).  So the
@@ -111,6 +113,9 @@ __device__ inline void fence_before() { asm volatile("tcgen05.fence::before_thre
 __device__ inline void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
 
 __device__ inline float tf32_hi(float x) { return __uint_as_float(__float_as_uint(x) & 0xffffe000u); }
+// lo part rounded to the nearest tf32 (the tensor core would truncate it,
+// a one-sided 2^-22 relative bias per correction term)
+__device__ inline float tf32_rn(float x) { return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xffffe000u); }
 
 __device__ inline void sts128(uint32_t addr, float a, float b, float c, float d) {
   asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "f"(a), "f"(b), "f"(c), "f"(d)
@@ -193,7 +198,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
         const uint32_t o = umma_off(rr, j, TM);
         const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
         sts128(a_hi + o, h0, h1, h2, h3);
-        sts128(a_lo + o, v.x - h0, v.y - h1, v.z - h2, v.w - h3);
+        sts128(a_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
       }
     } else {
       const uint8_t *sts = st_s + ((lt & 1) * 2 + b) * TM;
@@ -218,7 +223,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       const uint32_t o = umma_off(z, j, TS);
       const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
       sts128(b_hi + o, h0, h1, h2, h3);
-      sts128(b_lo + o, v.x - h0, v.y - h1, v.z - h2, v.w - h3);
+      sts128(b_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
     }
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
   };
