@@ -188,14 +188,33 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
     const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
     const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
     const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+    constexpr int NA = TM * 16 / kThr, NB = TS * 16 / kThr;  // 16-byte chunks per thread
+    float4 va[NA], vb[NB];
+    const float *P = static_cast<const float *>(b == 0 ? op.P1 : op.P2) + (size_t)c * TS * TS;
+    // ---- every global load of this phase in flight before the first shared store
     if (!tip) {
       const float *A = static_cast<const float *>(b == 0 ? op.in1 : op.in2) + ((size_t)c * p_pad + p0) * TS;
-      for (int i = tid; i < TM * 16; i += kThr) {
+#pragma unroll
+      for (int u = 0; u < NA; ++u) {
+        const int i = tid + u * kThr;
         const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-        const int j = kb * 2 + kh;
-        float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (p0 + rr < p) v = __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + j * 4));
-        const uint32_t o = umma_off(rr, j, TM);
+        va[u] = (p0 + rr < p) ? __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + (kb * 2 + kh) * 4))
+                              : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < NB; ++u) {  // natural [z][x] layout = K-major B
+      const int i = tid + u * kThr;
+      const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
+      vb[u] = __ldg(reinterpret_cast<const float4 *>(P + z * TS + (kb * 2 + kh) * 4));
+    }
+    if (!tip) {
+#pragma unroll
+      for (int u = 0; u < NA; ++u) {
+        const int i = tid + u * kThr;
+        const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
+        const uint32_t o = umma_off(rr, kb * 2 + kh, TM);
+        const float4 v = va[u];
         const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
         sts128(a_hi + o, h0, h1, h2, h3);
         sts128(a_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
@@ -215,12 +234,12 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
         sts128(a_hi + umma_off(rr, j, TM), v[0], v[1], v[2], v[3]);
       }
     }
-    const float *P = static_cast<const float *>(b == 0 ? op.P1 : op.P2) + (size_t)c * TS * TS;
-    for (int i = tid; i < TS * 16; i += kThr) {  // natural [z][x] layout = K-major B
+#pragma unroll
+    for (int u = 0; u < NB; ++u) {
+      const int i = tid + u * kThr;
       const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
-      const int j = kb * 2 + kh;
-      const float4 v = __ldg(reinterpret_cast<const float4 *>(P + z * TS + j * 4));
-      const uint32_t o = umma_off(z, j, TS);
+      const uint32_t o = umma_off(z, kb * 2 + kh, TS);
+      const float4 v = vb[u];
       const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
       sts128(b_hi + o, h0, h1, h2, h3);
       sts128(b_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
