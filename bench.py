@@ -250,13 +250,28 @@ def main():
     import torch
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
+    local = local % torch.cuda.device_count()  # (several ranks may share a GPU in wiring tests)
     torch.cuda.set_device(local)
     # a dedicated (capturable, non-legacy) stream for everything timed below
     torch.cuda.set_stream(torch.cuda.Stream())
     dist = None
+    backend = os.environ.get("RRL_DIST_BACKEND", "nccl")  # gloo: CPU-side test of the wiring
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+
+    def allreduce_(t, op=None):
+        """In-place all-reduce of a device tensor (NCCL on the device; gloo via host)."""
+        op = dist.ReduceOp.SUM if op is None else op
+        if backend == "nccl":
+            dist.all_reduce(t, op=op)
+        else:
+            h = t.cpu()
+            dist.all_reduce(h, op=op)
+            t.copy_(h)
 
     from paper_conf_ipps_ayresc18_b200 import build as _b
     _b.build()
@@ -272,7 +287,7 @@ def main():
         if dist is None:
             return x
         t = torch.tensor([x], dtype=torch.float64, device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        allreduce_(t, dist.ReduceOp.MAX)
         return float(t.item())
 
     def make(w, mode, precision, reuse):
@@ -292,7 +307,7 @@ def main():
         tl.update()
         tl.root_loglik_device(d_out.data_ptr())
         if dist is not None:
-            dist.all_reduce(d_out)
+            allreduce_(d_out)
 
     def timed(tl, steps, warmup):
         """Per-step CUDA events on the launching stream; L2 flushed before
@@ -415,7 +430,7 @@ def main():
         tl.update()
         tl.root_loglik_device(d_out.data_ptr())
         if dist is not None:
-            dist.all_reduce(d_out)
+            allreduce_(d_out)
         float(d_out.item())
     e2e_s = maxall(time.perf_counter() - t0)
     e2e_val = prim["fl"] * world * e2e_steps / e2e_s / 1e9
