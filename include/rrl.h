@@ -264,6 +264,24 @@ int rrl_reroot_and_schedule(int tip_count, const int32_t *parent, const double *
 int rrl_reroot_edge_table(int tip_count, const int32_t *parent, int32_t *out_key,
                           int32_t *out_sets, int32_t *out_imbalance);
 
+/* Partial-tree update schedule (host; only the part of
+ * the tree above a change is recomputed).  nodes[node_count]: the lowest
+ * internal nodes whose partials must be recomputed (e.g. parent(v) after the
+ * branch above v changed); every ancestor up to the root is added.  Writes
+ * the level-batched ops (same conventions as rrl_reroot_and_schedule, current
+ * rooting, identity buffers) to out_ops[<= n-1] and out_set_offsets[<= n];
+ * out_op_count / out_set_count receive the sizes.  Internal node ids only
+ * (RRL_ERROR_OUT_OF_RANGE otherwise). */
+int rrl_schedule_partial(int tip_count, const int32_t *parent, const int32_t *nodes, int node_count,
+                         rrl_op *out_ops, int32_t *out_set_offsets, int32_t *out_op_count,
+                         int32_t *out_set_count);
+
+/* The paper's exhaustive O(n^2) rerooting search in C++, with
+ * the same objective and tie-break as rrl_reroot_and_schedule's O(n) DP; for
+ * cost comparisons.  blen may be NULL. */
+int rrl_reroot_exhaustive(int tip_count, const int32_t *parent, const double *blen,
+                          int32_t *out_root_edge, int32_t *out_set_count);
+
 /* Substitution model (host, fp64): builds the normalised rate matrix Q
  * (-sum_i pi_i Q_ii = 1) for model in {"jc69","hky","gtr","gy94"} and its
  * eigensystem through the symmetric form S = Pi^1/2 Q Pi^-1/2 (cyclic Jacobi).

@@ -264,3 +264,105 @@ extern "C" int rrl_reroot_and_schedule(int tip_count, const int32_t *parent, con
     return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_reroot_and_schedule");
   }
 }
+
+// ---------------------------------------------------------------------------
+// Partial-tree updates (§VII-D, §VIII:
+// "phylogenetic analysis programs only calculate those subtree partial
+// likelihoods as required for a topology change").  The caller names the
+// lowest internal nodes whose partials must be recomputed (e.g. parent(v)
+// after v's branch length changed); the library adds every ancestor up to the
+// root and level-batches exactly those operations on the current rooting:
+// level(v) = 1 + max level of v's children that are recomputed (1 if none).
+extern "C" int rrl_schedule_partial(int tip_count, const int32_t *parent, const int32_t *nodes,
+                                    int node_count, rrl_op *out_ops, int32_t *out_set_offsets,
+                                    int32_t *out_op_count, int32_t *out_set_count) {
+  try {
+    View v;
+    int rc = build_view(tip_count, parent, v);
+    if (rc < 0) return rc;
+    const int n = v.n, N = v.N;
+    if (node_count < 0 || (node_count > 0 && !nodes)) return rrl::fail(RRL_ERROR_GENERAL, "nodes");
+    std::vector<char> mark(N, 0);
+    for (int i = 0; i < node_count; ++i) {
+      int x = nodes[i];
+      if (x < n || x >= N) return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "partial-update node must be internal");
+      while (x >= 0 && !mark[x]) {
+        mark[x] = 1;
+        x = v.parent[x];
+      }
+    }
+    std::vector<int> lev(N, 0);
+    int H = 0, cnt = 0;
+    for (int x : v.post)
+      if (mark[x]) {
+        int l = 0;
+        if (mark[v.c1[x]]) l = lev[v.c1[x]];
+        if (mark[v.c2[x]]) l = std::max(l, lev[v.c2[x]]);
+        lev[x] = l + 1;
+        H = std::max(H, lev[x]);
+        ++cnt;
+      }
+    std::vector<int> count(H + 2, 0), offs(H + 1, 0);
+    for (int x = n; x < N; ++x)
+      if (mark[x]) ++count[lev[x]];
+    for (int k = 1; k <= H; ++k) offs[k] = offs[k - 1] + count[k];
+    std::vector<int> fill(offs.begin(), offs.end()), order(cnt);
+    for (int x = n; x < N; ++x)
+      if (mark[x]) order[fill[lev[x] - 1]++] = x;
+    if (out_ops)
+      for (int i = 0; i < cnt; ++i) {
+        const int x = order[i];
+        out_ops[i] = rrl_op{x, x - n, RRL_NONE, v.c1[x], v.c1[x], v.c2[x], v.c2[x]};
+      }
+    if (out_set_offsets) std::copy(offs.begin(), offs.end(), out_set_offsets);
+    if (out_op_count) *out_op_count = cnt;
+    if (out_set_count) *out_set_count = H;
+    return RRL_SUCCESS;
+  } catch (...) {
+    return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_schedule_partial");
+  }
+}
+
+// ---------------------------------------------------------------------------
+// The paper's own search (§VI-E), in C++ for the cost comparison
+// of SURVEY.md NEXT-4: for every one of the 2n-3 edges, rebuild the rooted
+// tree there (path reversal) and measure its height; O(n^2).  Same tie-break
+// as the O(n) DP (reading A9); returns the chosen edge key, writes its set
+// count.
+extern "C" int rrl_reroot_exhaustive(int tip_count, const int32_t *parent, const double *blen,
+                                     int32_t *out_root_edge, int32_t *out_set_count) {
+  try {
+    View v;
+    int rc = build_view(tip_count, parent, v);
+    if (rc < 0) return rc;
+    const int n = v.n, N = v.N, R = v.root, a = v.c1[R], b = v.c2[R];
+    std::vector<double> zero;
+    if (!blen) zero.assign(N, 0.0);
+    const double *bl = blen ? blen : zero.data();
+    const int cur = std::min(a, b);
+    EdgeRow best{1 << 30, 1, 1 << 30, 1 << 30};
+    std::vector<int> par;
+    std::vector<double> nb;
+    std::vector<int> h(N), tips(N);
+    for (int key = 0; key < N; ++key) {
+      if (key == R || key == std::max(a, b)) continue;  // the merged root edge is keyed by min(a, b)
+      reroot(v, bl, key, par, nb);
+      View w;
+      rc = build_view(n, par.data(), w);
+      if (rc < 0) return rc;
+      std::fill(h.begin(), h.end(), 0);
+      std::fill(tips.begin(), tips.begin() + n, 1);
+      for (int x : w.post) {
+        h[x] = 1 + std::max(h[w.c1[x]], h[w.c2[x]]);
+        tips[x] = tips[w.c1[x]] + tips[w.c2[x]];
+      }
+      const EdgeRow row{h[w.root], key == cur ? 0 : 1, std::abs(tips[w.c1[w.root]] - tips[w.c2[w.root]]), key};
+      if (row < best) best = row;
+    }
+    if (out_root_edge) *out_root_edge = best.key;
+    if (out_set_count) *out_set_count = best.sets;
+    return RRL_SUCCESS;
+  } catch (...) {
+    return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_reroot_exhaustive");
+  }
+}

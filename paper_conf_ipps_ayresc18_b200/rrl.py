@@ -98,6 +98,8 @@ _SIGS = {
     "rrl_reroot_and_schedule": (_I, [_I, _P, _P, C.c_uint32, _P, _P, _P, _P, _P, _P, _P]),
     "rrl_reroot_edge_table": (_I, [_I, _P, _P, _P, _P]),
     "rrl_model_eigensystem": (_I, [C.c_char_p, _I, _P, _P, _I, _P, _P, _P, _P]),
+    "rrl_schedule_partial": (_I, [_I, _P, _P, _I, _P, _P, _P, _P]),
+    "rrl_reroot_exhaustive": (_I, [_I, _P, _P, _P, _P]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -341,3 +343,27 @@ def rrl_model_eigensystem(model: str, pi, params=()):
     _chk(_lib.rrl_model_eigensystem(model.encode(), s, _ptr(pi), _ptr(prm), len(params), _ptr(Q),
                                     _ptr(V), _ptr(Vi), _ptr(lam)), "rrl_model_eigensystem")
     return Q, V, Vi, lam
+
+
+def rrl_schedule_partial(tip_count, parent, nodes):
+    """Returns dict(ops (OP_DTYPE), set_offsets, op_count, set_count)."""
+    par = _c(parent, np.int32)
+    nd = _c(nodes, np.int32)
+    ops = np.empty(max(1, tip_count - 1), OP_DTYPE)
+    offs = np.empty(tip_count, np.int32)
+    nop = np.zeros(1, np.int32)
+    nset = np.zeros(1, np.int32)
+    _chk(_lib.rrl_schedule_partial(tip_count, _ptr(par), _ptr(nd), nd.shape[0], _ptr(ops), _ptr(offs),
+                                   _ptr(nop), _ptr(nset)), "rrl_schedule_partial")
+    k, m = int(nset[0]), int(nop[0])
+    return dict(ops=ops[:m].copy(), set_offsets=offs[: k + 1].copy(), op_count=m, set_count=k)
+
+
+def rrl_reroot_exhaustive(tip_count, parent, blen=None):
+    par = _c(parent, np.int32)
+    bl = None if blen is None else _c(blen, np.float64)
+    key = np.zeros(1, np.int32)
+    sets = np.zeros(1, np.int32)
+    _chk(_lib.rrl_reroot_exhaustive(tip_count, _ptr(par), _ptr(bl), _ptr(key), _ptr(sets)),
+         "rrl_reroot_exhaustive")
+    return int(key[0]), int(sets[0])

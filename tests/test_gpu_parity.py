@@ -424,3 +424,33 @@ def test_c4_full_size_sampled_patterns():
     np.testing.assert_allclose(site[idx], ora.site_lnl, rtol=1e-4)
     assert np.isfinite(total)
     tl.close()
+
+
+# ------------------------------------------------------------------ partial updates (NEXT-2)
+@pytest.mark.parametrize("precision", [64, 32])
+def test_partial_update_equals_full_recompute(precision):
+    """Change one branch length, recompute only the path to the root
+    (rrl_schedule_partial): bit-identical to a full pass."""
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="random", n=150, p=5_000, model="gtr", c=4, seed=31)
+    tl = gpu_setup(w, "reroot", precision)
+    tl.loglik()
+    rt = rooted(tl)
+    rng = np.random.default_rng(3)
+    for _ in range(3):
+        v = int(rng.choice(tl.matrix_idx))
+        new_t = float(rng.uniform(0.01, 0.3))
+        pos = int(np.flatnonzero(tl.matrix_idx == v)[0])
+        tl.t[pos] = new_t
+        R.rrl_update_transition_matrices(tl.inst, 0, np.array([v], np.int32), np.array([new_t]))
+        sch = R.rrl_schedule_partial(w.n, rt.parent, np.array([rt.parent[v]], np.int32))
+        R.rrl_update_partials(tl.inst, sch["ops"], sch["set_offsets"])
+        partial = tl.root_loglik()
+        full = tl.loglik()                    # K1 for all branches + every level set
+        assert partial == full
+        blen = rt.blen.copy()
+        blen[v] = new_t
+        rt = Tree(rt.n, rt.parent, blen)
+        ora = oracle_run(w, tree=rt)
+        assert rel(full, ora.lnl) <= LNL_TOL[precision]
+    tl.close()

@@ -149,3 +149,29 @@ def test_model_eigensystem_vs_oracle(R, name):
     np.testing.assert_allclose(V @ np.diag(lam) @ Vi, Qo, atol=1e-12)
     assert abs(np.sort(lam)[-1]) < 1e-12     # one zero eigenvalue, rest negative
     assert np.all(np.sort(lam)[:-1] < 0)
+
+
+@pytest.mark.parametrize("kind", ["random", "yule", "pectinate", "balanced"])
+def test_partial_schedule_matches_oracle(R, kind):
+    rng = np.random.default_rng(1)
+    for n in (3, 10, 64, 200):
+        t = make_tree(kind, n, seed=n)
+        for _ in range(5):
+            k = int(rng.integers(1, 4))
+            nodes = rng.integers(n, 2 * n - 1, size=k)
+            exp_ops, exp_offs = orr.schedule_partial(t, nodes.tolist())
+            got = R.rrl_schedule_partial(n, t.parent, nodes)
+            assert _ops_tuple(got["ops"]) == exp_ops
+            assert got["set_offsets"].tolist() == exp_offs
+    with pytest.raises(R.RRLError):
+        R.rrl_schedule_partial(5, make_tree("random", 5, seed=1).parent, np.array([2]))
+
+
+def test_exhaustive_cpp_equals_dp(R):
+    """The paper's O(n^2) search (C++) and the O(n) DP choose the same edge."""
+    for kind in ("random", "yule", "pectinate"):
+        for seed in range(1, 6):
+            t = make_tree(kind, 300, seed=seed)
+            key, sets = R.rrl_reroot_exhaustive(300, t.parent, t.blen)
+            g = R.rrl_reroot_and_schedule(300, t.parent, t.blen, "reroot")
+            assert key == g["root_edge"] and sets == g["set_count"]
