@@ -17,6 +17,10 @@ the sequential one-op-per-launch schedule), the 406-OTU pectinate point of
 PAPER.md:258 (best 1.93x on GP100), and Fig. 4/5 (100 paper-random 256-OTU
 trees: sets and throughput original vs rerooted; mean speedup 1.26x on GP100,
 PAPER.md:230).
+
+Part C (NEXT-4): host cost of the O(n) rerooting DP and of the paper's
+exhaustive O(n^2) search (C++) against the per-pass time rerooting saves
+(PAPER.md:270, 288).
 """
 from __future__ import annotations
 
@@ -163,6 +167,30 @@ def main():
                                     "paper": "mean 1.26x on Quadro GP100 (PAPER.md:230); sets reduced by "
                                              "up to half (PAPER.md:205)"}
     print(json.dumps({k: v for k, v in B["fig4_fig5_256otu_512pat"].items() if k != "trees"}), flush=True)
+    # ---------------- Part C (NEXT-4): cost of rerooting vs its benefit
+    C = []
+    for kind in ("random", "pectinate"):
+        for n in (64, 256, 1024, 4096):
+            w = make_workload(tree_kind=kind, n=n, p=512, model="gtr", c=4, seed=1)
+            reps = 20
+            t0 = time.perf_counter()
+            for _ in range(reps):
+                R.rrl_reroot_and_schedule(n, w.tree.parent, w.tree.blen, "reroot")
+            dp_ms = (time.perf_counter() - t0) / reps * 1e3
+            t0 = time.perf_counter()
+            R.rrl_reroot_exhaustive(n, w.tree.parent, w.tree.blen)
+            ex_ms = (time.perf_counter() - t0) * 1e3
+            o = run(w, "level", 32, 10)
+            r = run(w, "reroot", 32, 10)
+            saved = o["mean_ms"] - r["mean_ms"]
+            row = {"kind": kind, "n": n, "patterns": 512, "dp_reroot_schedule_ms": dp_ms,
+                   "exhaustive_cpp_ms": ex_ms, "pass_orig_ms": o["mean_ms"], "pass_reroot_ms": r["mean_ms"],
+                   "saved_per_pass_ms": saved,
+                   "breakeven_passes_dp": (dp_ms / saved) if saved > 0 else None,
+                   "breakeven_passes_exhaustive": (ex_ms / saved) if saved > 0 else None}
+            C.append(row)
+            print(json.dumps(row), flush=True)
+    out["partC_reroot_cost"] = C
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     json.dump(out, open(args.out, "w"), indent=1)
 
