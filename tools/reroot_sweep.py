@@ -5,8 +5,9 @@
 
 Part A (§8(d)-5): 1,024-tip pectinate, GTR+G4, fp32 and fp64, patterns in
 {512, 1K, 2K, 4K, 10K, 100K, 1M}: original-root (1,023 sets) vs rerooted (512
-sets) level-set schedules.  Reports, per point, the updatePartials time (sum
-of per-set durations from CUDA events inside the replayed CUDA graph), the
+sets) level-set schedules.  Reports, per point, the updatePartials time (CUDA
+events on the launching stream around each CUDA-graph replay of all level-set
+launches; L2 flushed before every replay), the
 reroot speedup S = T_orig / T_reroot against the bound 1,023/512, and the
 rerooted algorithmic-HBM fraction.
 
