@@ -543,7 +543,10 @@ int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cuda
   constexpr int U = 1;
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads * U - 1) / (kThreads * U));
-  // One wave: a second wave would double this launch's latency.
+  // At most half of the resident CTA slots: a second wave would double this
+  // launch's latency, and the free half lets the NEXT level set's CTAs become
+  // resident early (programmatic dependent launch) and sit in
+  // griddepcontrol.wait while this set drains.
   static int resident = -1;  // per template instance
   if (resident < 0) {
     int per_sm = 1, dev = 0, nsm = 148;
@@ -552,7 +555,7 @@ int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cuda
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     resident = (per_sm > 0 ? per_sm : 1) * nsm;
   }
-  int gx = resident / nops;
+  int gx = (resident / 2) / nops;
   if (gx > nchunks) gx = nchunks;
   if (gx < 1) gx = 1;
   for (int o = 0; o < nops; o += 65535) {
