@@ -538,24 +538,12 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
 }
 
 // ============================================================ host launchers
-template <typename T, int C>
-int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
-  constexpr int U = 1;
+template <typename T, int C, int U>
+int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int gx_cap,
+                     cudaStream_t st) {
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads * U - 1) / (kThreads * U));
-  // At most half of the resident CTA slots: a second wave would double this
-  // launch's latency, and the free half lets the NEXT level set's CTAs become
-  // resident early (programmatic dependent launch) and sit in
-  // griddepcontrol.wait while this set drains.
-  static int resident = -1;  // per template instance
-  if (resident < 0) {
-    int per_sm = 1, dev = 0, nsm = 148;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, U>, kThreads, 0);
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    resident = (per_sm > 0 ? per_sm : 1) * nsm;
-  }
-  int gx = (resident / 2) / nops;
+  int gx = gx_cap / nops;
   if (gx > nchunks) gx = nchunks;
   if (gx < 1) gx = 1;
   for (int o = 0; o < nops; o += 65535) {
@@ -579,6 +567,29 @@ int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cuda
     if (e != cudaSuccess) return (int)e;
   }
   return 0;
+}
+
+// Items per thread U: the smallest of 1, 2, 4 for which the whole set fits in
+// one round on at most half of the resident CTA slots (a second round doubles
+// the launch's latency; the free half lets the NEXT level set's CTAs become
+// resident early under programmatic dependent launch and wait in
+// griddepcontrol.wait); otherwise one full wave.
+template <typename T, int C>
+int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
+  static int resident = -1;  // per template instance
+  if (resident < 0) {
+    int per_sm = 1, dev = 0, nsm = 148;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, 4>, kThreads, 0);
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    resident = (per_sm > 0 ? per_sm : 1) * nsm;
+  }
+  const long long items = (long long)p * C;
+  auto ctas = [&](int u) { return (long long)nops * ((items + kThreads * u - 1) / (kThreads * u)); };
+  if (ctas(1) <= resident / 2) return launch_latency_u<T, C, 1>(d_ops, h_ops, nops, p, resident / 2, st);
+  if (ctas(2) <= resident / 2) return launch_latency_u<T, C, 2>(d_ops, h_ops, nops, p, resident / 2, st);
+  if (ctas(4) <= resident / 2) return launch_latency_u<T, C, 4>(d_ops, h_ops, nops, p, resident / 2, st);
+  return launch_latency_u<T, C, 1>(d_ops, h_ops, nops, p, resident, st);
 }
 
 template <typename T, int C>
