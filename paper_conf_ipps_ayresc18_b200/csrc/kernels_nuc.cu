@@ -569,26 +569,21 @@ int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, in
   return 0;
 }
 
-// Items per thread U: the smallest of 1, 2, 4 for which the whole set fits in
-// one round on at most half of the resident CTA slots (a second round doubles
-// the launch's latency; the free half lets the NEXT level set's CTAs become
-// resident early under programmatic dependent launch and wait in
-// griddepcontrol.wait); otherwise one full wave.
+// One item per thread and at most one full wave of resident CTAs: measured on
+// configs[1], fewer CTAs with more items per thread (leaving slots free for
+// the next level set's early PDL launch) is slower (0.29-0.41 ms vs 0.236 ms
+// per step): a launch this small is bound by its one dependent memory round
+// trip, so the widest single round wins.
 template <typename T, int C>
 int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
   static int resident = -1;  // per template instance
   if (resident < 0) {
     int per_sm = 1, dev = 0, nsm = 148;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, 4>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, 1>, kThreads, 0);
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     resident = (per_sm > 0 ? per_sm : 1) * nsm;
   }
-  const long long items = (long long)p * C;
-  auto ctas = [&](int u) { return (long long)nops * ((items + kThreads * u - 1) / (kThreads * u)); };
-  if (ctas(1) <= resident / 2) return launch_latency_u<T, C, 1>(d_ops, h_ops, nops, p, resident / 2, st);
-  if (ctas(2) <= resident / 2) return launch_latency_u<T, C, 2>(d_ops, h_ops, nops, p, resident / 2, st);
-  if (ctas(4) <= resident / 2) return launch_latency_u<T, C, 4>(d_ops, h_ops, nops, p, resident / 2, st);
   return launch_latency_u<T, C, 1>(d_ops, h_ops, nops, p, resident, st);
 }
 
