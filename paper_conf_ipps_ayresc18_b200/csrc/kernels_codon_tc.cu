@@ -179,49 +179,60 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       }
   };
 
-  // operands of phase g into buffer g & 1
-  auto build = [&](int g) {
+  // Operands of phase g: fetch(g) issues every global load of the phase into
+  // registers (fa / fb); stage(g) converts them (hi/lo split, or the one-hot
+  // rows of a tip child) into buffer g & 1 in the UMMA layout.  fetch runs a
+  // phase ahead of stage, so each phase's load latency hides behind the
+  // previous phase's conversion, MMA wait and epilogue.
+  constexpr int NA = TM * 16 / kThr, NB = TS * 16 / kThr;  // 16-byte chunks per thread
+  float4 fa[NA], fb[NB];
+  auto fetch = [&](int g) {
     const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
     const int f = blockIdx.x + lt * gridDim.x;
     const DevOp &op = ops[f / ntiles];
     const int p0 = (f % ntiles) * TM;
     const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
-    const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
-    const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
-    constexpr int NA = TM * 16 / kThr, NB = TS * 16 / kThr;  // 16-byte chunks per thread
-    float4 va[NA], vb[NB];
-    const float *P = static_cast<const float *>(b == 0 ? op.P1 : op.P2) + (size_t)c * TS * TS;
-    // ---- every global load of this phase in flight before the first shared store
     if (!tip) {
       const float *A = static_cast<const float *>(b == 0 ? op.in1 : op.in2) + ((size_t)c * p_pad + p0) * TS;
 #pragma unroll
       for (int u = 0; u < NA; ++u) {
         const int i = tid + u * kThr;
         const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-        va[u] = (p0 + rr < p) ? __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + (kb * 2 + kh) * 4))
+        fa[u] = (p0 + rr < p) ? __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + (kb * 2 + kh) * 4))
                               : make_float4(0.f, 0.f, 0.f, 0.f);
       }
     }
+    const float *P = static_cast<const float *>(b == 0 ? op.P1 : op.P2) + (size_t)c * TS * TS;
 #pragma unroll
     for (int u = 0; u < NB; ++u) {  // natural [z][x] layout = K-major B
       const int i = tid + u * kThr;
       const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
-      vb[u] = __ldg(reinterpret_cast<const float4 *>(P + z * TS + (kb * 2 + kh) * 4));
+      fb[u] = __ldg(reinterpret_cast<const float4 *>(P + z * TS + (kb * 2 + kh) * 4));
     }
+  };
+  auto stage = [&](int g) {
+    const int lt = g / (2 * C), b = g & 1;
+    const int f = blockIdx.x + lt * gridDim.x;
+    const DevOp &op = ops[f / ntiles];
+    const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+    const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
+    const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
     if (!tip) {
 #pragma unroll
       for (int u = 0; u < NA; ++u) {
         const int i = tid + u * kThr;
         const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
         const uint32_t o = umma_off(rr, kb * 2 + kh, TM);
-        const float4 v = va[u];
+        const float4 v = fa[u];
         const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
         sts128(a_hi + o, h0, h1, h2, h3);
         sts128(a_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
       }
     } else {
       const uint8_t *sts = st_s + ((lt & 1) * 2 + b) * TM;
-      for (int i = tid; i < TM * 16; i += kThr) {
+#pragma unroll
+      for (int u = 0; u < NA; ++u) {
+        const int i = tid + u * kThr;
         const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
         const int j = kb * 2 + kh;
         const unsigned sv = sts[rr];
@@ -239,7 +250,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       const int i = tid + u * kThr;
       const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
       const uint32_t o = umma_off(z, kb * 2 + kh, TS);
-      const float4 v = vb[u];
+      const float4 v = fb[u];
       const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
       sts128(b_hi + o, h0, h1, h2, h3);
       sts128(b_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
@@ -274,8 +285,10 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
 
   if (nphase > 0) {
     load_states(0);
+    fetch(0);
     __syncthreads();
-    build(0);
+    stage(0);
+    if (nphase > 1) fetch(1);
     fence_before();
     __syncthreads();
     if (tid == 0) {
@@ -290,7 +303,8 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
         load_states(lt + 1);
         __syncthreads();
       }
-      build(g + 1);  // overlaps the MMAs of phase g
+      stage(g + 1);                    // overlaps the MMAs of phase g
+      if (g + 2 < nphase) fetch(g + 2);  // in flight through the epilogue of phase g
     }
     bar_wait(bar, phase);
     phase ^= 1u;
