@@ -51,7 +51,7 @@ constexpr int kThr = 256;
 constexpr int A_BYTES = TM * TS * 4;  // 32 KB per operand tile
 constexpr int B_BYTES = TS * TS * 4;  // 16 KB
 constexpr int BUF_BYTES = 2 * A_BYTES + 2 * B_BYTES;  // A hi/lo + B hi/lo of one phase
-constexpr int S1_STRIDE = TS + 1;
+constexpr int S1_STRIDE = TS;  // rows of 16 x 16-byte chunks, chunk k stored at k ^ (row & 15)
 // smem: 2 operand buffers, child-1 result, tip states [tile parity][child][128],
 // row maxima [2 halves][128], mbarrier, TMEM base address
 constexpr int SMEM_BUF = 0;
@@ -328,50 +328,64 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
 #pragma unroll
       for (int i = 0; i < 16; ++i) d[half * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
     }
-    float *s1row = S1 + r * S1_STRIDE + h * 32;
+    // S1 chunk (row, k) lives at S1 + row*64 + 4*(k ^ (row & 15)): the 32 lanes
+    // (32 rows) of a row-per-lane access hit different banks
+    auto s1 = [&](int row, int k) -> float4 * {
+      return reinterpret_cast<float4 *>(S1 + row * S1_STRIDE + 4 * (k ^ (row & 15)));
+    };
     if (b == 0) {
 #pragma unroll
-      for (int i = 0; i < 32; ++i) s1row[i] = d[i];
+      for (int i = 0; i < 8; ++i) *s1(r, h * 8 + i) = make_float4(d[4 * i], d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
     } else {
       float *out = static_cast<float *>(op.out);
 #pragma unroll
-      for (int i = 0; i < 32; ++i) {
-        d[i] *= s1row[i];
-        m = fmaxf(m, d[i]);
+      for (int i = 0; i < 8; ++i) {  // product in place in S1, running max over (c, z)
+        float4 v = *s1(r, h * 8 + i);
+        v.x *= d[4 * i]; v.y *= d[4 * i + 1]; v.z *= d[4 * i + 2]; v.w *= d[4 * i + 3];
+        m = fmaxf(m, fmaxf(fmaxf(v.x, v.y), fmaxf(v.z, v.w)));
+        *s1(r, h * 8 + i) = v;
       }
-      if (valid) {
-        float4 *dst = reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + pp) * TS + h * 32);
+      __syncthreads();
+      // coalesced store of the (unscaled) category tile: a warp writes 2 whole rows
 #pragma unroll
-        for (int i = 0; i < 8; ++i) dst[i] = make_float4(d[4 * i], d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
+      for (int u = 0; u < TM * 16 / kThr; ++u) {
+        const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+        if (p0 + row < p)
+          *reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + p0 + row) * TS + ch * 4) =
+              *s1(row, ch);
       }
-      if (c == C - 1) {  // ---- tile done: exponent from max over (c, z), rescale own rows
+      if (c == C - 1) {  // ---- tile done: exponent from max over (c, z), coalesced rescale
         mx[h * TM + r] = m;
         __syncthreads();
-        const float mm = fmaxf(mx[r], mx[TM + r]);
-        int e = 0;
-        if (op.scale_out != nullptr) {
-          e = frexp_e(mm);
-          if (valid && h == 0) {
-            int tot = e;
-            if (op.cum1 != nullptr) tot += op.cum1[pp];
-            if (op.cum2 != nullptr) tot += op.cum2[pp];
-            op.scale_out[pp] = tot;
+        if (h == 0) {
+          const float mm = fmaxf(mx[r], mx[TM + r]);
+          int e = 0;
+          if (op.scale_out != nullptr) {
+            e = frexp_e(mm);
+            if (valid) {
+              int tot = e;
+              if (op.cum1 != nullptr) tot += op.cum1[pp];
+              if (op.cum2 != nullptr) tot += op.cum2[pp];
+              op.scale_out[pp] = tot;
+            }
+          } else if (op.scale_in != nullptr) {
+            e = valid ? op.scale_in[pp] : 0;
           }
-        } else if (op.scale_in != nullptr) {
-          e = valid ? op.scale_in[pp] : 0;
+          mx[r] = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
         }
-        if (valid && e != 0) {
-          const float sc = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
-          for (int cat = 0; cat < C; ++cat) {
-            float4 *row = reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + pp) * TS + h * 32);
+        __syncthreads();
+        for (int cat = 0; cat < C; ++cat)
 #pragma unroll
-            for (int i = 0; i < 8; ++i) {
-              float4 v = row[i];
+          for (int u = 0; u < TM * 16 / kThr; ++u) {
+            const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+            const float sc = mx[row];
+            if (p0 + row < p && sc != 1.f) {
+              float4 *q4 = reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4);
+              float4 v = *q4;
               v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
-              row[i] = v;
+              *q4 = v;
             }
           }
-        }
         m = 0.f;
       }
     }
