@@ -61,7 +61,8 @@ constexpr int SMEM_MX = SMEM_ST + 2 * 2 * TM;
 constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;
 constexpr int SMEM_TMEM = SMEM_BAR + 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 8;
-constexpr int kTmemCols = 512;  // 5 x 64 used (4 main + 1 correction accumulators)
+constexpr int kTmemCols = 512;  // 5 x 64 accumulator columns (4 main + 1 correction) ...
+constexpr int kProdCol = 5 * TS;  // ... then the parked unscaled products of categories 0..C-2
 
 __device__ inline uint32_t smem_addr(const void *p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -108,6 +109,16 @@ __device__ inline void tmem_ld16(uint32_t taddr, float (&v)[16]) {
 #pragma unroll
   for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
 }
+__device__ inline void tmem_st16(uint32_t taddr, const float *v) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(taddr),
+      "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])), "r"(__float_as_uint(v[3])),
+      "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])), "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])),
+      "r"(__float_as_uint(v[8])), "r"(__float_as_uint(v[9])), "r"(__float_as_uint(v[10])), "r"(__float_as_uint(v[11])),
+      "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])), "r"(__float_as_uint(v[14])), "r"(__float_as_uint(v[15]))
+      : "memory");
+}
+__device__ inline void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 __device__ inline void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 __device__ inline void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
 __device__ inline void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
@@ -135,6 +146,8 @@ __device__ inline int frexp_e(float m) {
 template <int C>
 __global__ void __launch_bounds__(kThr, 1)
 k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles, int total) {
+  // categories 0..C-2 wait in TMEM for the tile's exponent when they fit
+  constexpr bool kProdInTmem = kProdCol + (C - 1) * TS <= kTmemCols;
   extern __shared__ __align__(1024) unsigned char sm[];
   uint64_t *bar = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(sm + SMEM_TMEM);
@@ -339,22 +352,30 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
     } else {
       float *out = static_cast<float *>(op.out);
 #pragma unroll
-      for (int i = 0; i < 8; ++i) {  // product in place in S1, running max over (c, z)
-        float4 v = *s1(r, h * 8 + i);
-        v.x *= d[4 * i]; v.y *= d[4 * i + 1]; v.z *= d[4 * i + 2]; v.w *= d[4 * i + 3];
-        m = fmaxf(m, fmaxf(fmaxf(v.x, v.y), fmaxf(v.z, v.w)));
-        *s1(r, h * 8 + i) = v;
+      for (int i = 0; i < 8; ++i) {  // product, running max over (c, z)
+        const float4 v = *s1(r, h * 8 + i);
+        d[4 * i] *= v.x; d[4 * i + 1] *= v.y; d[4 * i + 2] *= v.z; d[4 * i + 3] *= v.w;
+        m = fmaxf(m, fmaxf(fmaxf(d[4 * i], d[4 * i + 1]), fmaxf(d[4 * i + 2], d[4 * i + 3])));
       }
-      __syncthreads();
-      // coalesced store of the (unscaled) category tile: a warp writes 2 whole rows
+      if constexpr (kProdInTmem) {
+        if (c < C - 1) {  // park the unscaled product in TMEM until the exponent is known
+          tmem_st16(tl + (uint32_t)(kProdCol + c * TS), d);
+          tmem_st16(tl + (uint32_t)(kProdCol + c * TS + 16), d + 16);
+          tmem_wait_st();
+        }
+      } else {
+        __syncthreads();  // S1 no longer read as child 1: stage the product for a coalesced store
 #pragma unroll
-      for (int u = 0; u < TM * 16 / kThr; ++u) {
-        const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
-        if (p0 + row < p)
-          *reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + p0 + row) * TS + ch * 4) =
-              *s1(row, ch);
+        for (int i = 0; i < 8; ++i) *s1(r, h * 8 + i) = make_float4(d[4 * i], d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
+        __syncthreads();
+#pragma unroll
+        for (int u = 0; u < TM * 16 / kThr; ++u) {
+          const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+          if (p0 + row < p)
+            *reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
+        }
       }
-      if (c == C - 1) {  // ---- tile done: exponent from max over (c, z), coalesced rescale
+      if (c == C - 1) {  // ---- tile done: exponent from max over (c, z)
         mx[h * TM + r] = m;
         __syncthreads();
         if (h == 0) {
@@ -374,18 +395,55 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
           mx[r] = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
         }
         __syncthreads();
-        for (int cat = 0; cat < C; ++cat)
+        if constexpr (kProdInTmem) {
+          // scaled categories through the swizzled shared tile, coalesced stores, written once
+          const float sc = mx[r];
+          for (int cat = 0; cat < C; ++cat) {
+            float v[32];
+            if (cat < C - 1) {
+              float lo16[16], hi16[16];
+              tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), lo16);
+              tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), hi16);
+              tmem_wait_ld();
 #pragma unroll
-          for (int u = 0; u < TM * 16 / kThr; ++u) {
-            const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
-            const float sc = mx[row];
-            if (p0 + row < p && sc != 1.f) {
-              float4 *q4 = reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4);
-              float4 v = *q4;
-              v.x *= sc; v.y *= sc; v.z *= sc; v.w *= sc;
-              *q4 = v;
+              for (int i = 0; i < 16; ++i) { v[i] = lo16[i]; v[16 + i] = hi16[i]; }
+            } else {
+#pragma unroll
+              for (int i = 0; i < 32; ++i) v[i] = d[i];
+            }
+            if (cat > 0) __syncthreads();  // previous category's tile fully read
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              *s1(r, h * 8 + i) = make_float4(v[4 * i] * sc, v[4 * i + 1] * sc, v[4 * i + 2] * sc, v[4 * i + 3] * sc);
+            __syncthreads();
+#pragma unroll
+            for (int u = 0; u < TM * 16 / kThr; ++u) {
+              const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+              if (p0 + row < p)
+                *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
             }
           }
+        } else {
+          // products already stored unscaled: coalesced in-place rescale (L2-resident)
+          for (int cat = 0; cat < C; ++cat) {
+            float4 v[TM * 16 / kThr];
+#pragma unroll
+            for (int u = 0; u < TM * 16 / kThr; ++u) {  // all loads first
+              const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+              v[u] = (p0 + row < p)
+                         ? *reinterpret_cast<const float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4)
+                         : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+#pragma unroll
+            for (int u = 0; u < TM * 16 / kThr; ++u) {
+              const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+              const float sc = mx[row];
+              if (p0 + row < p && sc != 1.f)
+                *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) =
+                    make_float4(v[u].x * sc, v[u].y * sc, v[u].z * sc, v[u].w * sc);
+            }
+          }
+        }
         m = 0.f;
       }
     }
