@@ -377,14 +377,20 @@ def main():
                                    "per-launch duration = region time / level-set launches"},
             "lnL": float(d_out.item()),
         }
-        if s == 61:
-            # SIMT codon kernel: bound by FP32/FP64 FMA issue, not HBM
-            peak_tf = 148 * 128 * 2 * 1.965e9 / 1e12 if precision == 32 else 148 * 64 * 2 * 1.965e9 / 1e12
+        if s == 61 and precision == 32:
+            # tcgen05 codon kernel: HBM-bound once the tensor cores carry the
+            # contraction; algorithmic bytes count 61 states (the 64-wide
+            # padding is overhead).  Tensor work for context.
+            res["roofline"]["tensor_tflops"] = fl / (part_ms * 1e-3) / 1e12
+            res["roofline"]["kernel"] = "k_partials_codon_tc (tcgen05 kind::tf32, 3xTF32)"
+        if s == 61 and precision == 64:
+            # SIMT fp64 codon kernel: bound by FP64 FMA issue, not HBM
+            peak_tf = 148 * 64 * 2 * 1.965e9 / 1e12
             ach = fl / (part_ms * 1e-3) / 1e12
             res["roofline"].update({
                 "bound": "alu", "achieved": ach, "peak": peak_tf, "unit": "TFLOP/s",
                 "frac": ach / peak_tf, "hbm_achieved_gbs": achieved,
-                "peak_source": "derived: 148 SMs x 128 FP32 (64 FP64) lanes x 2 flop x 1.965 GHz "
+                "peak_source": "derived: 148 SMs x 64 FP64 lanes x 2 flop x 1.965 GHz "
                                "(B200_PROFILING.md clocks; DESIGN.md §6)",
                 "flops": "effective Eq.(1) flops (n-1) c s (4s-1) per pattern (reading A16)"})
         if with_original and cfg != "c4":
