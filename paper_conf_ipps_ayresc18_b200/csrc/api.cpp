@@ -693,13 +693,18 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
     for (int k = 0; k < nsets; ++k) {
       const int n = offs[k + 1] - offs[k];
       Timed tm(I, 0, !capturing);  // eager profiling: one event pair per set launch
-      int e = (I->s == 4) ? launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k],
-                                                       I->h_ops + offs[k], n, I->p, I->p_pad, I->stream)
-                          : (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))
-                                ? launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, I->p, I->p_pad,
-                                                                  I->stream)
-                                : launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k],
-                                                               I->h_ops + offs[k], n, I->p, I->p_pad, I->stream);
+      int e;
+      if (I->s == 4) {
+        e = launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, I->p,
+                                       I->p_pad, I->stream);
+      } else {
+        e = (int)cudaErrorNotSupported;
+        if (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))  // tcgen05 path (c <= 4)
+          e = launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, I->p, I->p_pad, I->stream);
+        if (e == (int)cudaErrorNotSupported)
+          e = launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, I->p,
+                                           I->p_pad, I->stream);
+      }
       if (e == (int)cudaErrorNotSupported) return fail(RRL_ERROR_NO_IMPLEMENTATION, "kernel variant");
       if (e != 0) return fail(RRL_ERROR_CUDA, std::string("updatePartials launch: ") +
                                                   cudaGetErrorString(static_cast<cudaError_t>(e)));
