@@ -47,9 +47,9 @@ namespace {
 constexpr int TM = 128;  // patterns per tile = MMA M = TMEM lanes
 constexpr int TS = 64;   // padded states: MMA N and K
 constexpr int kS61 = 61;
-constexpr int kEpi = 128;             // warps 0-3: epilogue (TMEM lane quarters)
-constexpr int kProd = 128;            // warps 4-7: operand producers
-constexpr int kThr = kEpi + kProd + 32;  // + warp 8: MMA issuer
+constexpr int kEpi = 256;             // warps 0-7: epilogue (TMEM lane quarter x column half)
+constexpr int kProd = 128;            // warps 8-11: operand producers
+constexpr int kThr = kEpi + kProd + 32;  // + warp 12: MMA issuer
 constexpr int A_BYTES = TM * TS * 4;  // 32 KB per operand tile
 constexpr int B_BYTES = TS * TS * 4;  // 16 KB
 constexpr int BUF_BYTES = 2 * A_BYTES + 2 * B_BYTES;  // A hi/lo + B hi/lo of one phase
@@ -59,7 +59,8 @@ constexpr int S1_STRIDE = TS;  // rows of 16 x 16-byte chunks, chunk k stored at
 constexpr int SMEM_BUF = 0;
 constexpr int SMEM_S1 = 2 * BUF_BYTES;
 constexpr int SMEM_ST = SMEM_S1 + TM * S1_STRIDE * 4;
-constexpr int SMEM_BAR = SMEM_ST + 2 * TM;
+constexpr int SMEM_MX = SMEM_ST + 2 * TM;       // row maxima / scale factors [2][128]
+constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;
 constexpr int SMEM_TMEM = SMEM_BAR + 6 * 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 8;
 constexpr int kTmemCols = 512;    // 5 x 64 accumulator columns (4 main + 1 correction) ...
@@ -163,7 +164,7 @@ __device__ inline void named_sync(int id, int n) { asm volatile("bar.sync %0, %1
 //     product (parked in TMEM for categories < C-1); after the last category:
 //     exponent of the row, scale, coalesced stores through a swizzled tile.
 template <int C>
-__global__ void __launch_bounds__(kThr, 1)
+__global__ void __maxnreg__(152)
 k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles, int total) {
   static_assert(kProdCol + (C - 1) * TS <= kTmemCols, "parked products must fit TMEM");
   extern __shared__ __align__(1024) unsigned char sm[];
@@ -314,12 +315,17 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
     }
   } else {
     // =============================================================== epilogue
-    const int r = warp * 32 + lane;  // TMEM lane = pattern row of the tile
-    const uint32_t tl = tmem + ((uint32_t)(warp * 32) << 16);
+    // warp w: TMEM lane quarter w & 3 (one pattern row per thread), column
+    // half h = w >> 2 (32 of the 64 states): two warps per lane quarter
+    // double the tcgen05.ld throughput that paces the accumulator turnaround.
+    const int h = warp >> 2;
+    const int r = (warp & 3) * 32 + lane;
+    const uint32_t tl = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)(h * 32);
+    float *mx = reinterpret_cast<float *>(sm + SMEM_MX);
     auto s1 = [&](int row, int k) -> float4 * {
       return reinterpret_cast<float4 *>(S1 + row * S1_STRIDE + 4 * (k ^ (row & 15)));
     };
-    float m = 0.f;  // child 1 of the current category waits in this thread's own S1 row
+    float m = 0.f;  // child 1 of the current category waits in this thread's own S1 half-row
     for (int g = 0; g < nphase; ++g) {
       const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
       const int f = blockIdx.x + lt * gridDim.x;
@@ -329,9 +335,9 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       const bool valid = pp < p;
       bar_wait(acc_full, (uint32_t)g & 1u);
       fence_after();
-      float dv[TS];
+      float dv[32];
 #pragma unroll
-      for (int q = 0; q < TS / 16; ++q) {
+      for (int q = 0; q < 2; ++q) {
         float a0[16], a1[16], a2[16], a3[16], cc[16];
         tmem_ld16(tl + 0 * TS + q * 16, a0);
         tmem_ld16(tl + 1 * TS + q * 16, a1);
@@ -347,59 +353,66 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       if (lane == 0) mbar_arrive1(acc_empty);  // the MMAs of phase g+1 may overwrite them
       if (b == 0) {
 #pragma unroll
-        for (int k = 0; k < 16; ++k) *s1(r, k) = make_float4(dv[4 * k], dv[4 * k + 1], dv[4 * k + 2], dv[4 * k + 3]);
+        for (int k = 0; k < 8; ++k)
+          *s1(r, h * 8 + k) = make_float4(dv[4 * k], dv[4 * k + 1], dv[4 * k + 2], dv[4 * k + 3]);
         continue;
       }
 #pragma unroll
-      for (int k = 0; k < 16; ++k) {
-        const float4 w = *s1(r, k);
+      for (int k = 0; k < 8; ++k) {
+        const float4 w = *s1(r, h * 8 + k);
         dv[4 * k] *= w.x; dv[4 * k + 1] *= w.y; dv[4 * k + 2] *= w.z; dv[4 * k + 3] *= w.w;
         m = fmaxf(m, fmaxf(fmaxf(dv[4 * k], dv[4 * k + 1]), fmaxf(dv[4 * k + 2], dv[4 * k + 3])));
       }
       if (c < C - 1) {  // park the unscaled product in TMEM until the exponent is known
-#pragma unroll
-        for (int q = 0; q < TS / 16; ++q) tmem_st16(tl + (uint32_t)(kProdCol + c * TS + q * 16), dv + q * 16);
+        tmem_st16(tl + (uint32_t)(kProdCol + c * TS), dv);
+        tmem_st16(tl + (uint32_t)(kProdCol + c * TS + 16), dv + 16);
         tmem_wait_st();
         continue;
       }
-      // ---- tile done: exponent of this row (max over (c, z)), scale, store
-      int e = 0;
-      if (op.scale_out != nullptr) {
-        e = frexp_e(m);
-        if (valid) {
-          int tot = e;
-          if (op.cum1 != nullptr) tot += op.cum1[pp];
-          if (op.cum2 != nullptr) tot += op.cum2[pp];
-          op.scale_out[pp] = tot;
+      // ---- tile done: row exponent from max over (c, z) of both halves
+      mx[h * TM + r] = m;
+      named_sync(1, kEpi);
+      if (h == 0) {
+        const float mm = fmaxf(mx[r], mx[TM + r]);
+        int e = 0;
+        if (op.scale_out != nullptr) {
+          e = frexp_e(mm);
+          if (valid) {
+            int tot = e;
+            if (op.cum1 != nullptr) tot += op.cum1[pp];
+            if (op.cum2 != nullptr) tot += op.cum2[pp];
+            op.scale_out[pp] = tot;
+          }
+        } else if (op.scale_in != nullptr) {
+          e = valid ? op.scale_in[pp] : 0;
         }
-      } else if (op.scale_in != nullptr) {
-        e = valid ? op.scale_in[pp] : 0;
+        mx[r] = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
       }
-      const float sc = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
+      named_sync(1, kEpi);
+      const float sc = mx[r];
       float *out = static_cast<float *>(op.out);
       for (int cat = 0; cat < C; ++cat) {
-        float v[TS];
+        float v[32];
         if (cat < C - 1) {
+          float lo16[16], hi16[16];
+          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), lo16);
+          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), hi16);
+          tmem_wait_ld();
 #pragma unroll
-          for (int q = 0; q < TS / 16; ++q) {
-            float t16[16];
-            tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + q * 16), t16);
-            tmem_wait_ld();
-#pragma unroll
-            for (int i = 0; i < 16; ++i) v[q * 16 + i] = t16[i];
-          }
+          for (int i = 0; i < 16; ++i) { v[i] = lo16[i]; v[16 + i] = hi16[i]; }
         } else {
 #pragma unroll
-          for (int i = 0; i < TS; ++i) v[i] = dv[i];
+          for (int i = 0; i < 32; ++i) v[i] = dv[i];
         }
         named_sync(1, kEpi);  // staging tile free
 #pragma unroll
-        for (int k = 0; k < 16; ++k)
-          *s1(r, k) = make_float4(v[4 * k] * sc, v[4 * k + 1] * sc, v[4 * k + 2] * sc, v[4 * k + 3] * sc);
+        for (int k = 0; k < 8; ++k)
+          *s1(r, h * 8 + k) = make_float4(v[4 * k] * sc, v[4 * k + 1] * sc, v[4 * k + 2] * sc, v[4 * k + 3] * sc);
         named_sync(1, kEpi);
+        const int et = tid;  // 0..255
 #pragma unroll
         for (int u = 0; u < TM * 16 / kEpi; ++u) {  // coalesced: a warp writes 2 rows
-          const int i = r + u * kEpi, row = i >> 4, ch = i & 15;
+          const int i = et + u * kEpi, row = i >> 4, ch = i & 15;
           if (p0 + row < p)
             *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
         }
