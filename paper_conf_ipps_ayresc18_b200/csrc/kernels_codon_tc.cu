@@ -164,7 +164,7 @@ __device__ inline void named_sync(int id, int n) { asm volatile("bar.sync %0, %1
 //     product (parked in TMEM for categories < C-1); after the last category:
 //     exponent of the row, scale, coalesced stores through a swizzled tile.
 template <int C>
-__global__ void __maxnreg__(152)
+__global__ void __launch_bounds__(kThr, 1)
 k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles, int total) {
   static_assert(kProdCol + (C - 1) * TS <= kTmemCols, "parked products must fit TMEM");
   extern __shared__ __align__(1024) unsigned char sm[];
