@@ -79,8 +79,7 @@ extern "C" {
                                           level-set launches in a CUDA graph and
                                           replay it on later identical calls */
 #define RRL_FLAG_CODON_SIMT 0x4u       /* 61-state fp32: use the FP32 SIMT kernel
-                                          instead of the tcgen05 (3xTF32) one
-                                          (which covers category_count <= 4) */
+                                          instead of the tcgen05 (3xTF32) one */
 
 /* Schedule flags (rrl_reroot_and_schedule). Low byte = mode. */
 #define RRL_SCHED_SEQUENTIAL 1u  /* post-order, one op per set (Fig.2 upper) */

@@ -20,19 +20,19 @@
 //    ~2^-11-smaller hi*lo + lo*hi corrections to a fifth; the five meet in
 //    fp32 in the epilogue.  A tip child's A tile is one-hot (all ones for a
 //    missing state -> row sums), exact in tf32, so its lo*hi is skipped.
-//  * Warp specialisation (one 288-thread CTA per SM, it owns all of TMEM):
-//    phases (tile, category, child) flow from 4 producer warps (global loads,
-//    hi/lo split straight into the canonical no-swizzle K-major UMMA layout
-//    -- 8-row x 16-byte core matrices, LBO = 128 B, SBO = 256 B -- in a
-//    2-stage shared-memory ring, fence.proxy.async) through one MMA-issuing
-//    lane (tcgen05.mma + tcgen05.commit) to 4 epilogue warps, connected only
-//    by mbarriers (full/empty per stage, acc_full/acc_empty for TMEM), so
-//    loads, conversions, MMAs and epilogues of consecutive phases overlap.
-//  * Epilogue (one pattern row per thread, tcgen05.ld 32x32b.x16): child 1
-//    stays in registers, child 2 forms the product, which is parked in TMEM
-//    for categories < C-1 (C <= 4 fits); after the last category the row's
-//    exponent is known (max over (c, z) is thread-local), every category is
-//    scaled and written once, coalesced, through a swizzled shared tile.
+//  * Work is a pipeline of phases (tile, category, child): while the MMAs of
+//    phase k run, all 256 threads build phase k+1's operands (global loads,
+//    hi/lo split) into the other half of a double-buffered shared-memory ring,
+//    directly in the canonical no-swizzle K-major UMMA layout (8-row x 16-byte
+//    core matrices; LBO = 128 B between the two K halves, SBO = 256 B between
+//    8-row groups), published to the async proxy with fence.proxy.async; one
+//    thread issues the MMAs and tcgen05.commit's them to an mbarrier.
+//  * Epilogue of a phase: all 8 warps (warp w: TMEM lane quarter w%4, column
+//    half w/4) sum the five accumulators (tcgen05.ld 32x32b.x16).  Child 1's
+//    result is parked in shared memory; child 2's is multiplied with it,
+//    stored unscaled and folded into the running max over (c, z).  After the
+//    last category the two column halves exchange their maxima, and every
+//    thread rescales its own rows by the exact 2^-e (an L2-resident re-read).
 // Persistent CTAs (one per SM: 320 TMEM columns, ~225 KB of shared memory)
 // walk the flattened (operation, tile) space of the level set.
 #include <cuda_runtime.h>
@@ -47,23 +47,21 @@ namespace {
 constexpr int TM = 128;  // patterns per tile = MMA M = TMEM lanes
 constexpr int TS = 64;   // padded states: MMA N and K
 constexpr int kS61 = 61;
-constexpr int kEpi = 256;             // warps 0-7: epilogue (TMEM lane quarter x column half)
-constexpr int kProd = 128;            // warps 8-11: operand producers
-constexpr int kThr = kEpi + kProd + 32;  // + warp 12: MMA issuer
+constexpr int kThr = 256;
 constexpr int A_BYTES = TM * TS * 4;  // 32 KB per operand tile
 constexpr int B_BYTES = TS * TS * 4;  // 16 KB
 constexpr int BUF_BYTES = 2 * A_BYTES + 2 * B_BYTES;  // A hi/lo + B hi/lo of one phase
 constexpr int S1_STRIDE = TS;  // rows of 16 x 16-byte chunks, chunk k stored at k ^ (row & 15)
-// smem: 2-stage operand ring, epilogue staging tile, producer tip states
-// [child][128], mbarriers full[2] empty[2] acc_full acc_empty, TMEM address
+// smem: 2 operand buffers, child-1 result, tip states [tile parity][child][128],
+// row maxima [2 halves][128], mbarrier, TMEM base address
 constexpr int SMEM_BUF = 0;
 constexpr int SMEM_S1 = 2 * BUF_BYTES;
 constexpr int SMEM_ST = SMEM_S1 + TM * S1_STRIDE * 4;
-constexpr int SMEM_MX = SMEM_ST + 2 * TM;       // row maxima / scale factors [2][128]
+constexpr int SMEM_MX = SMEM_ST + 2 * 2 * TM;
 constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;
-constexpr int SMEM_TMEM = SMEM_BAR + 6 * 8;
+constexpr int SMEM_TMEM = SMEM_BAR + 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 8;
-constexpr int kTmemCols = 512;    // 5 x 64 accumulator columns (4 main + 1 correction) ...
+constexpr int kTmemCols = 512;  // 5 x 64 accumulator columns (4 main + 1 correction) ...
 constexpr int kProdCol = 5 * TS;  // ... then the parked unscaled products of categories 0..C-2
 
 __device__ inline uint32_t smem_addr(const void *p) {
@@ -145,36 +143,17 @@ __device__ inline int frexp_e(float m) {
   return e;
 }
 
-__device__ inline void mbar_init1(uint64_t *bar, unsigned count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(bar)), "r"(count));
-}
-__device__ inline void mbar_arrive1(uint64_t *bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_addr(bar)) : "memory");
-}
-__device__ inline void named_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
-
-// Warp-specialised tcgen05 codon kernel.  Phases g = (local tile, category c,
-// child b) flow through three roles connected by mbarriers:
-//   producers (warps 4-7): wait empty[g&1]; load child tile + P rows; split
-//     hi/lo into the UMMA layout of stage g&1; fence.proxy.async; arrive full[g&1]
-//   MMA issuer (warp 8, one lane): wait full[g&1] and acc_empty; 8 K-steps of
-//     main (4 accumulators) + correction MMAs; commit -> empty[g&1], acc_full
-//   epilogue (warps 0-3, one pattern row per thread): wait acc_full; sum the
-//     five accumulators; release acc_empty; child 1 -> registers, child 2 ->
-//     product (parked in TMEM for categories < C-1); after the last category:
-//     exponent of the row, scale, coalesced stores through a swizzled tile.
 template <int C>
 __global__ void __launch_bounds__(kThr, 1)
 k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles, int total) {
-  static_assert(kProdCol + (C - 1) * TS <= kTmemCols, "parked products must fit TMEM");
+  // categories 0..C-2 wait in TMEM for the tile's exponent when they fit
+  constexpr bool kProdInTmem = kProdCol + (C - 1) * TS <= kTmemCols;
   extern __shared__ __align__(1024) unsigned char sm[];
-  uint64_t *full = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);
-  uint64_t *empty = full + 2;
-  uint64_t *acc_full = full + 4;
-  uint64_t *acc_empty = full + 5;
+  uint64_t *bar = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(sm + SMEM_TMEM);
-  uint8_t *st_p = sm + SMEM_ST;
+  uint8_t *st_s = sm + SMEM_ST;
   float *S1 = reinterpret_cast<float *>(sm + SMEM_S1);
+  float *mx = reinterpret_cast<float *>(sm + SMEM_MX);
   const uint32_t sbase = smem_addr(sm);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
 
@@ -184,13 +163,8 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
                  "r"(kTmemCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
-  if (tid == kEpi + kProd) {
-    mbar_init1(&full[0], kProd / 32);
-    mbar_init1(&full[1], kProd / 32);
-    mbar_init1(&empty[0], 1);
-    mbar_init1(&empty[1], 1);
-    mbar_init1(acc_full, 1);
-    mbar_init1(acc_empty, kEpi / 32);
+  if (tid == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_addr(bar)));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   fence_before();
@@ -202,226 +176,284 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
   asm volatile("griddepcontrol.launch_dependents;" :::);
 
   const int my_tiles = total > (int)blockIdx.x ? (total - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
-  const int nphase = my_tiles * C * 2;
+  const int nphase = my_tiles * C * 2;  // phases (tile, category, child)
 
-  if (warp >= (kEpi + kProd) / 32) {
-    // =============================================================== MMA issuer
-    if (lane == 0) {
-      for (int g = 0; g < nphase; ++g) {
-        const int lt = g / (2 * C), b = g & 1;
-        const int f = blockIdx.x + lt * gridDim.x;
-        const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
-        bar_wait(&full[g & 1], (uint32_t)(g >> 1) & 1u);
-        bar_wait(acc_empty, (uint32_t)(g & 1) ^ 1u);
-        fence_after();
-        const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
-        const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+  // tip states of local tile lt (parity lt & 1)
+  auto load_states = [&](int lt) {
+    const int f = blockIdx.x + lt * gridDim.x;
+    const DevOp &op = ops[f / ntiles];
+    const int p0 = (f % ntiles) * TM;
+    const void *in[2] = {op.in1, op.in2};
+    const int fl[2] = {op.flags & OP_TIP1, op.flags & OP_TIP2};
+    for (int b = 0; b < 2; ++b)
+      if (fl[b] && tid < TM) {
+        const int pp = p0 + tid;
+        st_s[((lt & 1) * 2 + b) * TM + tid] = pp < p ? static_cast<const uint8_t *>(in[b])[pp] : (uint8_t)kS61;
+      }
+  };
+
+  // Operands of phase g: fetch(g) issues every global load of the phase into
+  // registers (fa / fb); stage(g) converts them (hi/lo split, or the one-hot
+  // rows of a tip child) into buffer g & 1 in the UMMA layout.  fetch runs a
+  // phase ahead of stage, so each phase's load latency hides behind the
+  // previous phase's conversion, MMA wait and epilogue.
+  constexpr int NA = TM * 16 / kThr, NB = TS * 16 / kThr;  // 16-byte chunks per thread
+  float4 fa[NA], fb[NB];
+  auto fetch = [&](int g) {
+    const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
+    const int f = blockIdx.x + lt * gridDim.x;
+    const DevOp &op = ops[f / ntiles];
+    const int p0 = (f % ntiles) * TM;
+    const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+    if (!tip) {
+      const float *A = static_cast<const float *>(b == 0 ? op.in1 : op.in2) + ((size_t)c * p_pad + p0) * TS;
 #pragma unroll
-        for (int kb = 0; kb < TS / 8; ++kb) {
-          const uint64_t ah = umma_desc(a_hi + kb * (TM * 32)), al = umma_desc(a_lo + kb * (TM * 32));
-          const uint64_t bh = umma_desc(b_hi + kb * (TS * 32)), bl = umma_desc(b_lo + kb * (TS * 32));
-          const uint32_t dmain = tmem + (uint32_t)((kb >> 1) * TS), dcorr = tmem + (uint32_t)(4 * TS);
-          mma_tf32(dmain, ah, bh, (kb & 1) ? 1u : 0u);
-          mma_tf32(dcorr, ah, bl, kb > 0 ? 1u : 0u);
-          if (!tip) mma_tf32(dcorr, al, bh, 1u);
-        }
-        mma_commit(&empty[g & 1]);  // operand stage free once these MMAs completed
-        mma_commit(acc_full);       // accumulators ready for the epilogue
+      for (int u = 0; u < NA; ++u) {
+        const int i = tid + u * kThr;
+        const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
+        fa[u] = (p0 + rr < p) ? __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + (kb * 2 + kh) * 4))
+                              : make_float4(0.f, 0.f, 0.f, 0.f);
       }
     }
-  } else if (warp >= kEpi / 32) {
-    // =============================================================== producers
-    const int pt = tid - kEpi;
-    int cur_tile = -1;
-    for (int g = 0; g < nphase; ++g) {
-      const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
-      const int f = blockIdx.x + lt * gridDim.x;
-      const DevOp &op = ops[f / ntiles];
-      const int p0 = (f % ntiles) * TM;
-      if (lt != cur_tile) {  // the tile's tip states (both children)
-        named_sync(2, kProd);  // every producer is done with the previous tile's states
-        const uint8_t *s1p = static_cast<const uint8_t *>(op.in1), *s2p = static_cast<const uint8_t *>(op.in2);
-        const int pp = p0 + pt;
-        st_p[pt] = ((op.flags & OP_TIP1) && pp < p) ? s1p[pp] : (uint8_t)kS61;
-        st_p[TM + pt] = ((op.flags & OP_TIP2) && pp < p) ? s2p[pp] : (uint8_t)kS61;
-        named_sync(2, kProd);
-        cur_tile = lt;
-      }
-      const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
-      constexpr int NA = TM * 16 / kProd, NB = TS * 16 / kProd;  // 16-byte chunks per thread
-      float4 fa[NA], fb[NB];
-      // all global loads of the phase first (they overlap the wait for the stage)
-      if (!tip) {
-        const float *A = static_cast<const float *>(b == 0 ? op.in1 : op.in2) + ((size_t)c * p_pad + p0) * TS;
+    const float *P = static_cast<const float *>(b == 0 ? op.P1 : op.P2) + (size_t)c * TS * TS;
 #pragma unroll
-        for (int u = 0; u < NA; ++u) {
-          const int i = pt + u * kProd;
-          const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-          fa[u] = (p0 + rr < p) ? __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + (kb * 2 + kh) * 4))
-                                : make_float4(0.f, 0.f, 0.f, 0.f);
-        }
-      }
-      const float *P = static_cast<const float *>(b == 0 ? op.P1 : op.P2) + (size_t)c * TS * TS;
+    for (int u = 0; u < NB; ++u) {  // natural [z][x] layout = K-major B
+      const int i = tid + u * kThr;
+      const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
+      fb[u] = __ldg(reinterpret_cast<const float4 *>(P + z * TS + (kb * 2 + kh) * 4));
+    }
+  };
+  auto stage = [&](int g) {
+    const int lt = g / (2 * C), b = g & 1;
+    const int f = blockIdx.x + lt * gridDim.x;
+    const DevOp &op = ops[f / ntiles];
+    const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+    const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
+    const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+    if (!tip) {
 #pragma unroll
-      for (int u = 0; u < NB; ++u) {  // natural [z][x] layout = K-major B
-        const int i = pt + u * kProd;
-        const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
-        fb[u] = __ldg(reinterpret_cast<const float4 *>(P + z * TS + (kb * 2 + kh) * 4));
-      }
-      bar_wait(&empty[g & 1], ((uint32_t)(g >> 1) & 1u) ^ 1u);  // MMAs of phase g-2 done
-      const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
-      const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
-      if (!tip) {
-#pragma unroll
-        for (int u = 0; u < NA; ++u) {
-          const int i = pt + u * kProd;
-          const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-          const uint32_t o = umma_off(rr, kb * 2 + kh, TM);
-          const float4 v = fa[u];
-          const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
-          sts128(a_hi + o, h0, h1, h2, h3);
-          sts128(a_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
-        }
-      } else {
-        const uint8_t *sts = st_p + b * TM;
-#pragma unroll
-        for (int u = 0; u < NA; ++u) {
-          const int i = pt + u * kProd;
-          const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-          const int j = kb * 2 + kh;
-          const unsigned sv = sts[rr];
-          float v[4];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            const unsigned k = (unsigned)(j * 4 + q);
-            v[q] = (sv < (unsigned)kS61) ? (k == sv ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
-          }
-          sts128(a_hi + umma_off(rr, j, TM), v[0], v[1], v[2], v[3]);
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < NB; ++u) {
-        const int i = pt + u * kProd;
-        const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
-        const uint32_t o = umma_off(z, kb * 2 + kh, TS);
-        const float4 v = fb[u];
+      for (int u = 0; u < NA; ++u) {
+        const int i = tid + u * kThr;
+        const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
+        const uint32_t o = umma_off(rr, kb * 2 + kh, TM);
+        const float4 v = fa[u];
         const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
-        sts128(b_hi + o, h0, h1, h2, h3);
-        sts128(b_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
+        sts128(a_hi + o, h0, h1, h2, h3);
+        sts128(a_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
       }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
-      __syncwarp();
-      if (lane == 0) mbar_arrive1(&full[g & 1]);
+    } else {
+      const uint8_t *sts = st_s + ((lt & 1) * 2 + b) * TM;
+#pragma unroll
+      for (int u = 0; u < NA; ++u) {
+        const int i = tid + u * kThr;
+        const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
+        const int j = kb * 2 + kh;
+        const unsigned sv = sts[rr];
+        float v[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          const unsigned k = (unsigned)(j * 4 + q);
+          v[q] = (sv < (unsigned)kS61) ? (k == sv ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
+        }
+        sts128(a_hi + umma_off(rr, j, TM), v[0], v[1], v[2], v[3]);
+      }
     }
-  } else {
-    // =============================================================== epilogue
-    // warp w: TMEM lane quarter w & 3 (one pattern row per thread), column
-    // half h = w >> 2 (32 of the 64 states): two warps per lane quarter
-    // double the tcgen05.ld throughput that paces the accumulator turnaround.
-    const int h = warp >> 2;
-    const int r = (warp & 3) * 32 + lane;
-    const uint32_t tl = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)(h * 32);
-    float *mx = reinterpret_cast<float *>(sm + SMEM_MX);
+#pragma unroll
+    for (int u = 0; u < NB; ++u) {
+      const int i = tid + u * kThr;
+      const int kh = i & 1, z = (i >> 1) & (TS - 1), kb = i >> 7;
+      const uint32_t o = umma_off(z, kb * 2 + kh, TS);
+      const float4 v = fb[u];
+      const float h0 = tf32_hi(v.x), h1 = tf32_hi(v.y), h2 = tf32_hi(v.z), h3 = tf32_hi(v.w);
+      sts128(b_hi + o, h0, h1, h2, h3);
+      sts128(b_lo + o, tf32_rn(v.x - h0), tf32_rn(v.y - h1), tf32_rn(v.z - h2), tf32_rn(v.w - h3));
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
+  };
+
+  // single thread: the MMAs of phase g (operands in buffer g & 1)
+  auto issue = [&](int g) {
+    const int lt = g / (2 * C), b = g & 1;
+    const int f = blockIdx.x + lt * gridDim.x;
+    const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+    const uint32_t a_hi = sbase + SMEM_BUF + (g & 1) * BUF_BYTES, a_lo = a_hi + A_BYTES;
+    const uint32_t b_hi = a_hi + 2 * A_BYTES, b_lo = b_hi + B_BYTES;
+#pragma unroll
+    for (int kb = 0; kb < TS / 8; ++kb) {
+      const uint64_t ah = umma_desc(a_hi + kb * (TM * 32)), al = umma_desc(a_lo + kb * (TM * 32));
+      const uint64_t bh = umma_desc(b_hi + kb * (TS * 32)), bl = umma_desc(b_lo + kb * (TS * 32));
+      const uint32_t dmain = tmem + (uint32_t)((kb >> 1) * TS), dcorr = tmem + (uint32_t)(4 * TS);
+      mma_tf32(dmain, ah, bh, (kb & 1) ? 1u : 0u);
+      mma_tf32(dcorr, ah, bl, kb > 0 ? 1u : 0u);
+      if (!tip) mma_tf32(dcorr, al, bh, 1u);
+    }
+    mma_commit(bar);
+  };
+
+  const int q = warp & 3, h = warp >> 2;  // TMEM lane quarter, column half
+  const int r = q * 32 + lane;            // this thread's row (pattern) in the tile
+  const uint32_t tl = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(h * 32);
+  float m = 0.f;
+  uint32_t phase = 0;
+
+  if (nphase > 0) {
+    load_states(0);
+    fetch(0);
+    __syncthreads();
+    stage(0);
+    if (nphase > 1) fetch(1);
+    fence_before();
+    __syncthreads();
+    if (tid == 0) {
+      fence_after();
+      issue(0);
+    }
+  }
+  for (int g = 0; g < nphase; ++g) {
+    const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
+    if (g + 1 < nphase) {
+      if ((g + 1) % (2 * C) == 0) {  // next phase starts a new tile: its tip states
+        load_states(lt + 1);
+        __syncthreads();
+      }
+      stage(g + 1);                    // overlaps the MMAs of phase g
+      if (g + 2 < nphase) fetch(g + 2);  // in flight through the epilogue of phase g
+    }
+    bar_wait(bar, phase);
+    phase ^= 1u;
+    fence_after();
+    // ---- epilogue of phase g
+    const int f = blockIdx.x + lt * gridDim.x;
+    const DevOp &op = ops[f / ntiles];
+    const int p0 = (f % ntiles) * TM;
+    const int pp = p0 + r;
+    const bool valid = pp < p;
+    float d[32];
+#pragma unroll
+    for (int half = 0; half < 2; ++half) {
+      float a0[16], a1[16], a2[16], a3[16], cc[16];
+      tmem_ld16(tl + 0 * TS + half * 16, a0);
+      tmem_ld16(tl + 1 * TS + half * 16, a1);
+      tmem_ld16(tl + 2 * TS + half * 16, a2);
+      tmem_ld16(tl + 3 * TS + half * 16, a3);
+      tmem_ld16(tl + 4 * TS + half * 16, cc);
+      tmem_wait_ld();
+#pragma unroll
+      for (int i = 0; i < 16; ++i) d[half * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
+    }
+    // S1 chunk (row, k) lives at S1 + row*64 + 4*(k ^ (row & 15)): the 32 lanes
+    // (32 rows) of a row-per-lane access hit different banks
     auto s1 = [&](int row, int k) -> float4 * {
       return reinterpret_cast<float4 *>(S1 + row * S1_STRIDE + 4 * (k ^ (row & 15)));
     };
-    float m = 0.f;  // child 1 of the current category waits in this thread's own S1 half-row
-    for (int g = 0; g < nphase; ++g) {
-      const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
-      const int f = blockIdx.x + lt * gridDim.x;
-      const DevOp &op = ops[f / ntiles];
-      const int p0 = (f % ntiles) * TM;
-      const int pp = p0 + r;
-      const bool valid = pp < p;
-      bar_wait(acc_full, (uint32_t)g & 1u);
-      fence_after();
-      float dv[32];
+    if (b == 0) {
 #pragma unroll
-      for (int q = 0; q < 2; ++q) {
-        float a0[16], a1[16], a2[16], a3[16], cc[16];
-        tmem_ld16(tl + 0 * TS + q * 16, a0);
-        tmem_ld16(tl + 1 * TS + q * 16, a1);
-        tmem_ld16(tl + 2 * TS + q * 16, a2);
-        tmem_ld16(tl + 3 * TS + q * 16, a3);
-        tmem_ld16(tl + 4 * TS + q * 16, cc);
-        tmem_wait_ld();
-#pragma unroll
-        for (int i = 0; i < 16; ++i) dv[q * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
-      }
-      fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive1(acc_empty);  // the MMAs of phase g+1 may overwrite them
-      if (b == 0) {
-#pragma unroll
-        for (int k = 0; k < 8; ++k)
-          *s1(r, h * 8 + k) = make_float4(dv[4 * k], dv[4 * k + 1], dv[4 * k + 2], dv[4 * k + 3]);
-        continue;
-      }
-#pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const float4 w = *s1(r, h * 8 + k);
-        dv[4 * k] *= w.x; dv[4 * k + 1] *= w.y; dv[4 * k + 2] *= w.z; dv[4 * k + 3] *= w.w;
-        m = fmaxf(m, fmaxf(fmaxf(dv[4 * k], dv[4 * k + 1]), fmaxf(dv[4 * k + 2], dv[4 * k + 3])));
-      }
-      if (c < C - 1) {  // park the unscaled product in TMEM until the exponent is known
-        tmem_st16(tl + (uint32_t)(kProdCol + c * TS), dv);
-        tmem_st16(tl + (uint32_t)(kProdCol + c * TS + 16), dv + 16);
-        tmem_wait_st();
-        continue;
-      }
-      // ---- tile done: row exponent from max over (c, z) of both halves
-      mx[h * TM + r] = m;
-      named_sync(1, kEpi);
-      if (h == 0) {
-        const float mm = fmaxf(mx[r], mx[TM + r]);
-        int e = 0;
-        if (op.scale_out != nullptr) {
-          e = frexp_e(mm);
-          if (valid) {
-            int tot = e;
-            if (op.cum1 != nullptr) tot += op.cum1[pp];
-            if (op.cum2 != nullptr) tot += op.cum2[pp];
-            op.scale_out[pp] = tot;
-          }
-        } else if (op.scale_in != nullptr) {
-          e = valid ? op.scale_in[pp] : 0;
-        }
-        mx[r] = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
-      }
-      named_sync(1, kEpi);
-      const float sc = mx[r];
+      for (int i = 0; i < 8; ++i) *s1(r, h * 8 + i) = make_float4(d[4 * i], d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
+    } else {
       float *out = static_cast<float *>(op.out);
-      for (int cat = 0; cat < C; ++cat) {
-        float v[32];
-        if (cat < C - 1) {
-          float lo16[16], hi16[16];
-          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), lo16);
-          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), hi16);
-          tmem_wait_ld();
 #pragma unroll
-          for (int i = 0; i < 16; ++i) { v[i] = lo16[i]; v[16 + i] = hi16[i]; }
-        } else {
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = dv[i];
+      for (int i = 0; i < 8; ++i) {  // product, running max over (c, z)
+        const float4 v = *s1(r, h * 8 + i);
+        d[4 * i] *= v.x; d[4 * i + 1] *= v.y; d[4 * i + 2] *= v.z; d[4 * i + 3] *= v.w;
+        m = fmaxf(m, fmaxf(fmaxf(d[4 * i], d[4 * i + 1]), fmaxf(d[4 * i + 2], d[4 * i + 3])));
+      }
+      if constexpr (kProdInTmem) {
+        if (c < C - 1) {  // park the unscaled product in TMEM until the exponent is known
+          tmem_st16(tl + (uint32_t)(kProdCol + c * TS), d);
+          tmem_st16(tl + (uint32_t)(kProdCol + c * TS + 16), d + 16);
+          tmem_wait_st();
         }
-        named_sync(1, kEpi);  // staging tile free
+      } else {
+        __syncthreads();  // S1 no longer read as child 1: stage the product for a coalesced store
 #pragma unroll
-        for (int k = 0; k < 8; ++k)
-          *s1(r, h * 8 + k) = make_float4(v[4 * k] * sc, v[4 * k + 1] * sc, v[4 * k + 2] * sc, v[4 * k + 3] * sc);
-        named_sync(1, kEpi);
-        const int et = tid;  // 0..255
+        for (int i = 0; i < 8; ++i) *s1(r, h * 8 + i) = make_float4(d[4 * i], d[4 * i + 1], d[4 * i + 2], d[4 * i + 3]);
+        __syncthreads();
 #pragma unroll
-        for (int u = 0; u < TM * 16 / kEpi; ++u) {  // coalesced: a warp writes 2 rows
-          const int i = et + u * kEpi, row = i >> 4, ch = i & 15;
+        for (int u = 0; u < TM * 16 / kThr; ++u) {
+          const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
           if (p0 + row < p)
-            *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
+            *reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
         }
       }
-      named_sync(1, kEpi);  // staging reads done before rows are reused for child 1
-      m = 0.f;
+      if (c == C - 1) {  // ---- tile done: exponent from max over (c, z)
+        mx[h * TM + r] = m;
+        __syncthreads();
+        if (h == 0) {
+          const float mm = fmaxf(mx[r], mx[TM + r]);
+          int e = 0;
+          if (op.scale_out != nullptr) {
+            e = frexp_e(mm);
+            if (valid) {
+              int tot = e;
+              if (op.cum1 != nullptr) tot += op.cum1[pp];
+              if (op.cum2 != nullptr) tot += op.cum2[pp];
+              op.scale_out[pp] = tot;
+            }
+          } else if (op.scale_in != nullptr) {
+            e = valid ? op.scale_in[pp] : 0;
+          }
+          mx[r] = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
+        }
+        __syncthreads();
+        if constexpr (kProdInTmem) {
+          // scaled categories through the swizzled shared tile, coalesced stores, written once
+          const float sc = mx[r];
+          for (int cat = 0; cat < C; ++cat) {
+            float v[32];
+            if (cat < C - 1) {
+              float lo16[16], hi16[16];
+              tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), lo16);
+              tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), hi16);
+              tmem_wait_ld();
+#pragma unroll
+              for (int i = 0; i < 16; ++i) { v[i] = lo16[i]; v[16 + i] = hi16[i]; }
+            } else {
+#pragma unroll
+              for (int i = 0; i < 32; ++i) v[i] = d[i];
+            }
+            if (cat > 0) __syncthreads();  // previous category's tile fully read
+#pragma unroll
+            for (int i = 0; i < 8; ++i)
+              *s1(r, h * 8 + i) = make_float4(v[4 * i] * sc, v[4 * i + 1] * sc, v[4 * i + 2] * sc, v[4 * i + 3] * sc);
+            __syncthreads();
+#pragma unroll
+            for (int u = 0; u < TM * 16 / kThr; ++u) {
+              const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+              if (p0 + row < p)
+                *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
+            }
+          }
+        } else {
+          // products already stored unscaled: coalesced in-place rescale (L2-resident)
+          for (int cat = 0; cat < C; ++cat) {
+            float4 v[TM * 16 / kThr];
+#pragma unroll
+            for (int u = 0; u < TM * 16 / kThr; ++u) {  // all loads first
+              const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+              v[u] = (p0 + row < p)
+                         ? *reinterpret_cast<const float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4)
+                         : make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+#pragma unroll
+            for (int u = 0; u < TM * 16 / kThr; ++u) {
+              const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
+              const float sc = mx[row];
+              if (p0 + row < p && sc != 1.f)
+                *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) =
+                    make_float4(v[u].x * sc, v[u].y * sc, v[u].z * sc, v[u].w * sc);
+            }
+          }
+        }
+        m = 0.f;
+      }
+    }
+    fence_before();
+    __syncthreads();  // TMEM accumulators read, S1 / maxima settled, phase g+1 operands visible
+    if (g + 1 < nphase && tid == 0) {
+      fence_after();
+      issue(g + 1);
     }
   }
-  fence_before();
   __syncthreads();
   if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
 }
@@ -456,7 +488,7 @@ int launch_tc(const DevOp *d_ops, int nops, int p, int p_pad, cudaStream_t st) {
 
 }  // namespace
 
-// fp32 codon instances, c in {1, 2, 4}; cudaErrorNotSupported otherwise
+// fp32 codon instances, c in {1, 2, 4, 8}; cudaErrorNotSupported otherwise
 // (the caller then uses the SIMT kernel).
 int launch_update_partials_codon_tc(int c, const DevOp *d_ops, int nops, int p, int p_pad, void *stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
@@ -464,7 +496,8 @@ int launch_update_partials_codon_tc(int c, const DevOp *d_ops, int nops, int p, 
     case 1: return launch_tc<1>(d_ops, nops, p, p_pad, st);
     case 2: return launch_tc<2>(d_ops, nops, p, p_pad, st);
     case 4: return launch_tc<4>(d_ops, nops, p, p_pad, st);
-    default: return (int)cudaErrorNotSupported;  // c = 8: products do not fit TMEM -> SIMT
+    case 8: return launch_tc<8>(d_ops, nops, p, p_pad, st);
+    default: return (int)cudaErrorNotSupported;
   }
 }
 

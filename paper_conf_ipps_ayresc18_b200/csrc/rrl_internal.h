@@ -40,7 +40,7 @@ int launch_update_partials_nuc(int prec, int c, const DevOp *d_ops, const DevOp 
                                int p, int p_pad, void *stream);
 int launch_update_partials_codon(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
                                  int p, int p_pad, void *stream);
-// tcgen05 (tf32, 3xTF32) codon kernel: fp32, c in {1,2,4}; cudaErrorNotSupported otherwise.
+// tcgen05 (tf32, 3xTF32) codon kernel: fp32, c in {1,2,4,8}; cudaErrorNotSupported otherwise.
 int launch_update_partials_codon_tc(int c, const DevOp *d_ops, int nops, int p, int p_pad, void *stream);
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
