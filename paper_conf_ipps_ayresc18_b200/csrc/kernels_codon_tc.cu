@@ -133,6 +133,19 @@ __device__ inline void sts128(uint32_t addr, float a, float b, float c, float d)
                : "memory");
 }
 
+#ifdef RRL_TC_TRACE
+// dev-only phase timeline of CTA 0, thread 0 (tools/microbench/codon_tc_trace.cu)
+__device__ long long g_tc_trace[256][5];
+#define TC_TRACE(g, k)                                                      \
+  do {                                                                      \
+    if (blockIdx.x == 0 && threadIdx.x == 0 && (g) < 256) g_tc_trace[g][k] = clock64(); \
+  } while (0)
+#else
+#define TC_TRACE(g, k) \
+  do {                 \
+  } while (0)
+#endif
+
 __device__ inline int frexp_e(float m) {
   const unsigned b = __float_as_uint(m);
   const int eb = (int)((b >> 23) & 0xffu);
@@ -311,6 +324,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
   }
   for (int g = 0; g < nphase; ++g) {
     const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
+    TC_TRACE(g, 0);
     if (g + 1 < nphase) {
       if ((g + 1) % (2 * C) == 0) {  // next phase starts a new tile: its tip states
         load_states(lt + 1);
@@ -319,9 +333,11 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       stage(g + 1);                    // overlaps the MMAs of phase g
       if (g + 2 < nphase) fetch(g + 2);  // in flight through the epilogue of phase g
     }
+    TC_TRACE(g, 1);
     bar_wait(bar, phase);
     phase ^= 1u;
     fence_after();
+    TC_TRACE(g, 2);
     // ---- epilogue of phase g
     const int f = blockIdx.x + lt * gridDim.x;
     const DevOp &op = ops[f / ntiles];
@@ -447,8 +463,10 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
         m = 0.f;
       }
     }
+    TC_TRACE(g, 3);
     fence_before();
     __syncthreads();  // TMEM accumulators read, S1 / maxima settled, phase g+1 operands visible
+    TC_TRACE(g, 4);
     if (g + 1 < nphase && tid == 0) {
       fence_after();
       issue(g + 1);
