@@ -454,3 +454,27 @@ def test_partial_update_equals_full_recompute(precision):
         ora = oracle_run(w, tree=rt)
         assert rel(full, ora.lnl) <= LNL_TOL[precision]
     tl.close()
+
+
+# ------------------------------------------------------------------ stored-factor rescaling (A6)
+@pytest.mark.parametrize("kind,p,model,precision", [("yule", 3_000, "gtr", 32), ("yule", 20_000, "gtr", 64),
+                                                    ("random", 300, "gy94", 32), ("random", 200, "gy94", 64)])
+def test_dest_scale_read_reuses_factors(kind, p, model, precision):
+    """The paper's timed regime computes new factors once per 1,000 passes and
+    reuses them otherwise (reading A6).  Per-node mode:
+    pass 1 writes own exponents; pass 2 applies them (dest_scale_read) and must
+    reproduce every node bit for bit."""
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind=kind, n=40, p=p, model=model, c=4, seed=17)
+    tl = gpu_setup(w, "reroot", precision, cumulative=False)
+    first = tl.loglik()
+    nodes = [int(d) for d in tl.ops["dest"]]
+    before = {v: tl.partials(v) for v in nodes[::7]}
+    ops2 = tl.ops.copy()
+    ops2["dest_scale_read"] = ops2["dest_scale_write"]
+    ops2["dest_scale_write"] = -1
+    R.rrl_update_partials(tl.inst, ops2, tl.offsets)
+    for v, L in before.items():
+        np.testing.assert_array_equal(tl.partials(v), L)
+    assert tl.root_loglik() == first
+    tl.close()
