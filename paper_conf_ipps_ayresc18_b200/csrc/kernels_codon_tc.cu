@@ -412,8 +412,15 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
         }
         __syncthreads();
         if constexpr (kProdInTmem) {
-          // scaled categories through the swizzled shared tile, coalesced stores, written once
+          // scaled categories staged all at once -- slot 0..2 in the operand
+          // buffer MMA(g) has finished with, slot C-1 in S1 -- then coalesced
+          // stores: one barrier for the tile instead of two per category
           const float sc = mx[r];
+          float *slot_base = reinterpret_cast<float *>(sm + SMEM_BUF + (g & 1) * BUF_BYTES);
+          auto slot = [&](int cat, int row, int k) -> float4 * {
+            float *bse = (cat == C - 1) ? S1 : slot_base + cat * TM * TS;
+            return reinterpret_cast<float4 *>(bse + row * S1_STRIDE + 4 * (k ^ (row & 15)));
+          };
           for (int cat = 0; cat < C; ++cat) {
             float v[32];
             if (cat < C - 1) {
@@ -427,18 +434,18 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
 #pragma unroll
               for (int i = 0; i < 32; ++i) v[i] = d[i];
             }
-            if (cat > 0) __syncthreads();  // previous category's tile fully read
 #pragma unroll
             for (int i = 0; i < 8; ++i)
-              *s1(r, h * 8 + i) = make_float4(v[4 * i] * sc, v[4 * i + 1] * sc, v[4 * i + 2] * sc, v[4 * i + 3] * sc);
-            __syncthreads();
+              *slot(cat, r, h * 8 + i) = make_float4(v[4 * i] * sc, v[4 * i + 1] * sc, v[4 * i + 2] * sc, v[4 * i + 3] * sc);
+          }
+          __syncthreads();
+          for (int cat = 0; cat < C; ++cat)
 #pragma unroll
             for (int u = 0; u < TM * 16 / kThr; ++u) {
               const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
               if (p0 + row < p)
-                *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
+                *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *slot(cat, row, ch);
             }
-          }
         } else {
           // products already stored unscaled: coalesced in-place rescale (L2-resident)
           for (int cat = 0; cat < C; ++cat) {
