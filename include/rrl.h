@@ -71,6 +71,10 @@ extern "C" {
 
 #define RRL_NONE (-1)
 
+/* Pattern ranges of rrl_update_partials_ranged start at multiples of this
+ * (whole bulk-copy chunks); pad partitions with zero-weight patterns. */
+#define RRL_PATTERN_RANGE_ALIGN 512
+
 /* Instance flags (rrl_create_instance). */
 #define RRL_FLAG_SCALE_CUMULATIVE 0x1u /* dest scale = own exponent + children's
                                           (child scale buffer = child - tip_count);
@@ -164,6 +168,11 @@ int rrl_set_pattern_weights(int inst, const double *w /*[p]*/);
 int rrl_set_state_frequencies(int inst, int idx, const double *pi /*[s]*/);
 int rrl_set_category_rates(int inst, const double *r /*[c]*/);
 int rrl_set_category_weights(int inst, int idx, const double *w /*[c]*/);
+/* Category rates of model slot idx (0 <= idx < eigen_count) for partitioned
+ * analyses ("independent model parameters for each of these
+ * different subsets"); rrl_set_category_rates sets every slot.  K1 uses the
+ * rates of the slot passed as eigen_idx. */
+int rrl_set_category_rates_idx(int inst, int idx, const double *r /*[c]*/);
 
 /* --------------------------------------------------- transition matrices (K1)
  * P_{m,c} = V diag(exp(lambda * r_c * t_m)) Vinv for each listed matrix m and
@@ -189,6 +198,18 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count,
                         const int32_t *set_offsets /*[set_count+1] or NULL*/,
                         int set_count);
 
+/* Pattern-partition concurrency (§IV-A, "a multi-operation
+ * kernel ... to compute multiple likelihood arrays in a single execution
+ * launch, and use pointer arithmetic to allow different input and output
+ * arrays for different execution blocks"): like rrl_update_partials, but
+ * operation i only covers patterns [pattern_ranges[2i], pattern_ranges[2i+1]).
+ * Operations of different partitions (disjoint ranges, each with its own
+ * transition matrices) may share a set and a destination buffer, so a level
+ * set of every partition runs as ONE launch.  Range starts must be multiples
+ * of RRL_PATTERN_RANGE_ALIGN (RRL_ERROR_GENERAL otherwise). */
+int rrl_update_partials_ranged(int inst, const rrl_op *ops, const int32_t *pattern_ranges /*[2*op_count]*/,
+                               int op_count, const int32_t *set_offsets, int set_count);
+
 /* ------------------------------------------------------------ scaling (K5)
  * cumulative[p] += sum_k scale[scale_idx[k]][p]  (int32, exact). */
 int rrl_accumulate_scale_factors(int inst, const int32_t *scale_idx, int count,
@@ -208,6 +229,13 @@ int rrl_calculate_root_log_likelihoods(int inst, int root_buffer, int cat_weight
 int rrl_calculate_root_log_likelihoods_device(int inst, int root_buffer, int cat_weights_idx,
                                               int freqs_idx, int cumulative_idx,
                                               double *d_out);
+
+/* Root log-likelihood of the patterns [pattern_begin, pattern_end) only (one
+ * partition of a partitioned analysis; per-pattern values for that range are
+ * updated for rrl_get_site_log_likelihoods). */
+int rrl_calculate_root_log_likelihoods_range(int inst, int root_buffer, int cat_weights_idx,
+                                             int freqs_idx, int cumulative_idx, int pattern_begin,
+                                             int pattern_end, double *out_sum);
 
 /* ------------------------------------------------------------- edge (K6)
  * lnL_i = ln( sum_c w_c sum_z pi_z Lp[i][c][z] sum_x P_m[c][z][x] Lc[i][c][x] )

@@ -50,7 +50,7 @@ struct Instance {
   char *d_P = nullptr;                   // [n_mat][c][s_pad][s_pad]
   int32_t *d_scale = nullptr;            // [n_scale][p_pad]
   double *d_eig = nullptr;               // [n_eig][2 s^2 + s]
-  double *d_rates = nullptr;             // [c]
+  double *d_rates = nullptr;             // [n_eig][c] (per model / partition)
   double *d_catw = nullptr;              // [n_eig][c]
   double *d_freqs = nullptr;             // [n_eig][s]
   double *d_pw = nullptr;                // [p]
@@ -76,6 +76,7 @@ struct Instance {
   cudaEvent_t staging_ev = nullptr;
   std::vector<rrl_op> last_ops;
   std::vector<int32_t> last_offs;
+  std::vector<int32_t> last_ranges;
   bool ops_valid = false;
   cudaGraphExec_t graph = nullptr;       // replay of the set launches
   cudaStream_t graph_stream = nullptr;
@@ -332,7 +333,7 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
   CKC(cudaMemset(I->d_scale, 0, std::max<size_t>((size_t)scale_buffer_count * I->p_pad * 4, 256)));
   const size_t eig_sz = 2 * (size_t)state_count * state_count + state_count;
   CKC(cudaMalloc(&I->d_eig, sizeof(double) * eig_sz * eigen_count));
-  CKC(cudaMalloc(&I->d_rates, sizeof(double) * category_count));
+  CKC(cudaMalloc(&I->d_rates, sizeof(double) * category_count * eigen_count));
   CKC(cudaMalloc(&I->d_catw, sizeof(double) * category_count * eigen_count));
   CKC(cudaMalloc(&I->d_freqs, sizeof(double) * state_count * eigen_count));
   CKC(cudaMalloc(&I->d_pw, sizeof(double) * I->p_pad));
@@ -343,7 +344,7 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
   CKC(cudaMemset(I->d_count, 0, sizeof(unsigned)));
   CKC(cudaMallocHost(&I->h_out, sizeof(double)));
   {
-    std::vector<double> ones(I->p_pad, 1.0), r(category_count, 1.0),
+    std::vector<double> ones(I->p_pad, 1.0), r((size_t)category_count * eigen_count, 1.0),
         w((size_t)category_count * eigen_count, 1.0 / category_count),
         f((size_t)state_count * eigen_count, 1.0 / state_count);
     CKC(cudaMemcpy(I->d_pw, ones.data(), sizeof(double) * I->p, cudaMemcpyHostToDevice));
@@ -481,7 +482,19 @@ int rrl_set_state_frequencies(int inst, int idx, const double *pi) {
 int rrl_set_category_rates(int inst, const double *r) {
   GET(I, inst);
   if (!r) return fail(RRL_ERROR_GENERAL, "rates NULL");
-  CK(cudaMemcpyAsync(I->d_rates, r, sizeof(double) * I->c, cudaMemcpyHostToDevice, I->stream));
+  for (int idx = 0; idx < I->n_eig; ++idx)  // every model slot
+    CK(cudaMemcpyAsync(I->d_rates + (size_t)idx * I->c, r, sizeof(double) * I->c, cudaMemcpyHostToDevice,
+                       I->stream));
+  CK(cudaStreamSynchronize(I->stream));
+  return RRL_SUCCESS;
+}
+
+int rrl_set_category_rates_idx(int inst, int idx, const double *r) {
+  GET(I, inst);
+  if (idx < 0 || idx >= I->n_eig) return fail(RRL_ERROR_OUT_OF_RANGE, "rates index");
+  if (!r) return fail(RRL_ERROR_GENERAL, "rates NULL");
+  CK(cudaMemcpyAsync(I->d_rates + (size_t)idx * I->c, r, sizeof(double) * I->c, cudaMemcpyHostToDevice,
+                     I->stream));
   CK(cudaStreamSynchronize(I->stream));
   return RRL_SUCCESS;
 }
@@ -539,7 +552,8 @@ int rrl_update_transition_matrices(int inst, int eigen_idx, const int32_t *matri
   {
     Timed tm(I, 1);
     CKL(launch_transition_matrices(I->prec, I->s, I->s_pad, I->c, I->d_eig + eig_sz * eigen_idx,
-                                   I->d_rates, I->d_midx, I->d_t, count, I->d_P, I->stream));
+                                   I->d_rates + (size_t)eigen_idx * I->c, I->d_midx, I->d_t, count, I->d_P,
+                                   I->stream));
   }
   I->prof.matrices_launches += (count + 65534) / 65535;
   I->prof.kernel_launches += (count + 65534) / 65535;
@@ -584,9 +598,30 @@ int rrl_get_transition_matrix(int inst, int idx, double *out) {
   return RRL_SUCCESS;
 }
 
+static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *ranges, int op_count,
+                                const int32_t *set_offsets, int set_count);
+
 int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t *set_offsets,
                         int set_count) {
   GET(I, inst);
+  return update_partials_impl(I, ops, nullptr, op_count, set_offsets, set_count);
+}
+
+int rrl_update_partials_ranged(int inst, const rrl_op *ops, const int32_t *pattern_ranges, int op_count,
+                               const int32_t *set_offsets, int set_count) {
+  GET(I, inst);
+  if (op_count > 0 && !pattern_ranges) return fail(RRL_ERROR_GENERAL, "pattern_ranges NULL");
+  for (int i = 0; i < op_count; ++i) {
+    const int b = pattern_ranges[2 * i], e = pattern_ranges[2 * i + 1];
+    if (b < 0 || e > I->p || b >= e) return fail(RRL_ERROR_OUT_OF_RANGE, "pattern range");
+    if (b % RRL_PATTERN_RANGE_ALIGN != 0)
+      return fail(RRL_ERROR_GENERAL, "pattern range must start at a multiple of RRL_PATTERN_RANGE_ALIGN");
+  }
+  return update_partials_impl(I, ops, pattern_ranges, op_count, set_offsets, set_count);
+}
+
+static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *ranges, int op_count,
+                                const int32_t *set_offsets, int set_count) {
   if (op_count < 0 || (op_count > 0 && !ops)) return fail(RRL_ERROR_GENERAL, "ops");
   if (op_count == 0) return RRL_SUCCESS;
   const bool cumulative = (I->flags & RRL_FLAG_SCALE_CUMULATIVE) != 0;
@@ -618,8 +653,10 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
   }
   const int nsets = (int)offs.size() - 1;
 
+  std::vector<int32_t> rng;
+  if (ranges) rng.assign(ranges, ranges + 2 * op_count);
   const bool same = I->ops_valid && I->last_ops.size() == (size_t)op_count &&
-                    I->last_offs == offs &&
+                    I->last_offs == offs && I->last_ranges == rng &&
                     std::memcmp(I->last_ops.data(), ops, sizeof(rrl_op) * op_count) == 0;
   if (!same) {
     // --- validate
@@ -638,7 +675,7 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
         for (int ch : {o.child1, o.child2})
           if (ch < I->n_tips && !I->has_states[ch] && !I->tip_partials[ch])
             return fail(RRL_ERROR_GENERAL, "tip without data");
-        if (stamp[o.dest] == k) return fail(RRL_ERROR_GENERAL, "two ops write one buffer in a set");
+        if (stamp[o.dest] == k && !ranges) return fail(RRL_ERROR_GENERAL, "two ops write one buffer in a set");
         stamp[o.dest] = k;
         if (cumulative && o.dest_scale_write >= 0) {
           if (o.dest_scale_write != o.dest - I->n_tips)
@@ -678,12 +715,31 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
                        ? I->d_scale + (size_t)o.dest_scale_read * I->p_pad
                        : nullptr;
       if (!d.scale_out) d.cum1 = d.cum2 = nullptr;
+      // pattern range: every pointer is advanced to the range's first pattern
+      // (the partials' pattern stride is c*s_pad elements for 4 states, s_pad
+      // within each category plane for 61 states)
+      const int pb = ranges ? ranges[2 * i] : 0;
+      d.p = ranges ? ranges[2 * i + 1] - pb : I->p;
+      if (pb > 0) {
+        const size_t pel = (I->s == 4 ? (size_t)I->c * 4 : (size_t)I->s_pad) * pb * I->elt;
+        auto adv = [&](const void *q, bool tip) -> const void * {
+          return static_cast<const char *>(q) + (tip ? (size_t)pb : pel);
+        };
+        d.in1 = adv(d.in1, d.flags & OP_TIP1);
+        d.in2 = adv(d.in2, d.flags & OP_TIP2);
+        d.out = const_cast<void *>(adv(d.out, false));
+        if (d.scale_out) d.scale_out += pb;
+        if (d.scale_in) d.scale_in += pb;
+        if (d.cum1) d.cum1 += pb;
+        if (d.cum2) d.cum2 += pb;
+      }
       I->h_ops[i] = d;
     }
     CK(cudaMemcpyAsync(I->d_ops, I->h_ops, sizeof(DevOp) * op_count, cudaMemcpyHostToDevice, I->stream));
     CK(cudaEventRecord(I->staging_ev, I->stream));
     I->last_ops.assign(ops, ops + op_count);
     I->last_offs = offs;
+    I->last_ranges = rng;
     I->ops_valid = true;
     int rg = drop_graphs(I);
     if (rg < 0) return rg;
@@ -692,17 +748,22 @@ int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t
   auto launch_all = [&](bool capturing) -> int {
     for (int k = 0; k < nsets; ++k) {
       const int n = offs[k + 1] - offs[k];
+      int pmax = I->p;  // widest pattern range of the set (grids are sized for it)
+      if (ranges) {
+        pmax = 0;
+        for (int i = offs[k]; i < offs[k + 1]; ++i) pmax = std::max(pmax, ranges[2 * i + 1] - ranges[2 * i]);
+      }
       Timed tm(I, 0, !capturing);  // eager profiling: one event pair per set launch
       int e;
       if (I->s == 4) {
-        e = launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, I->p,
+        e = launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax,
                                        I->p_pad, I->stream);
       } else {
         e = (int)cudaErrorNotSupported;
         if (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))  // tcgen05 path (c <= 4)
-          e = launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, I->p, I->p_pad, I->stream);
+          e = launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, pmax, I->p_pad, I->stream);
         if (e == (int)cudaErrorNotSupported)
-          e = launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, I->p,
+          e = launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax,
                                            I->p_pad, I->stream);
       }
       if (e == (int)cudaErrorNotSupported) return fail(RRL_ERROR_NO_IMPLEMENTATION, "kernel variant");
@@ -795,7 +856,9 @@ int rrl_get_scale_factors(int inst, int idx, int32_t *out) {
 }
 
 static int root_common(Instance *I, int root_buffer, int cat_weights_idx, int freqs_idx,
-                       int cumulative_idx, double *d_out) {
+                       int cumulative_idx, double *d_out, int pb = 0, int pe = -1) {
+  if (pe < 0) pe = I->p;
+  if (pb < 0 || pe > I->p || pb >= pe) return fail(RRL_ERROR_OUT_OF_RANGE, "pattern range");
   if (root_buffer < 0 || root_buffer >= I->n_buf) return fail(RRL_ERROR_OUT_OF_RANGE, "root buffer");
   if (cat_weights_idx < 0 || cat_weights_idx >= I->n_eig || freqs_idx < 0 || freqs_idx >= I->n_eig)
     return fail(RRL_ERROR_OUT_OF_RANGE, "weights/freqs index");
@@ -803,12 +866,16 @@ static int root_common(Instance *I, int root_buffer, int cat_weights_idx, int fr
     return fail(RRL_ERROR_OUT_OF_RANGE, "cumulative index");
   const void *root = buffer_ptr(I, root_buffer);
   if (!root) return fail(RRL_ERROR_GENERAL, "root buffer has no partials");
-  const int32_t *cum = cumulative_idx >= 0 ? I->d_scale + (size_t)cumulative_idx * I->p_pad : nullptr;
+  const int32_t *cum = cumulative_idx >= 0 ? I->d_scale + (size_t)cumulative_idx * I->p_pad + pb : nullptr;
+  const size_t pel = (I->s == 4 ? (size_t)I->c * 4 : (size_t)I->s_pad) * pb * I->elt;
+  const int np = pe - pb;
+  const int nb = std::max(1, std::min(I->nblocks, (np + 255) / 256));
   {
     Timed tm(I, 2);
-    CKL(launch_root_lnl(I->prec, I->s, I->s_pad, I->c, root, I->d_catw + (size_t)cat_weights_idx * I->c,
-                        I->d_freqs + (size_t)freqs_idx * I->s, cum, I->d_pw, I->p, I->p_pad, I->d_site,
-                        I->d_block, I->d_count, I->nblocks, d_out, I->stream));
+    CKL(launch_root_lnl(I->prec, I->s, I->s_pad, I->c, static_cast<const char *>(root) + pel,
+                        I->d_catw + (size_t)cat_weights_idx * I->c, I->d_freqs + (size_t)freqs_idx * I->s, cum,
+                        I->d_pw + pb, np, I->p_pad, I->d_site + pb, I->d_block, I->d_count, nb, d_out,
+                        I->stream));
   }
   I->prof.root_launches += 1;
   I->prof.kernel_launches += 1;
@@ -866,6 +933,21 @@ int rrl_calculate_edge_log_likelihoods(int inst, int parent_buffer, int child_bu
   }
   I->prof.root_launches += 1;
   I->prof.kernel_launches += 1;
+  CK(cudaMemcpyAsync(I->h_out, I->d_out, sizeof(double), cudaMemcpyDeviceToHost, I->stream));
+  CK(cudaStreamSynchronize(I->stream));
+  *out_sum = *I->h_out;
+  if (!std::isfinite(*out_sum)) return fail(RRL_ERROR_FLOATING_POINT, "non-finite log-likelihood");
+  return RRL_SUCCESS;
+}
+
+int rrl_calculate_root_log_likelihoods_range(int inst, int root_buffer, int cat_weights_idx, int freqs_idx,
+                                             int cumulative_idx, int pattern_begin, int pattern_end,
+                                             double *out_sum) {
+  GET(I, inst);
+  if (!out_sum) return fail(RRL_ERROR_GENERAL, "out NULL");
+  int r = root_common(I, root_buffer, cat_weights_idx, freqs_idx, cumulative_idx, I->d_out, pattern_begin,
+                      pattern_end);
+  if (r < 0) return r;
   CK(cudaMemcpyAsync(I->h_out, I->d_out, sizeof(double), cudaMemcpyDeviceToHost, I->stream));
   CK(cudaStreamSynchronize(I->stream));
   *out_sum = *I->h_out;

@@ -76,6 +76,8 @@ k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
   extern __shared__ __align__(16) unsigned char smem_raw3[];
   CodonSmem<T> &sm = *reinterpret_cast<CodonSmem<T> *>(smem_raw3);
   const DevOp &op = ops[blockIdx.y];
+  p = op.p;  // this operation's pattern range (the grid covers the widest of the set)
+  if ((int)blockIdx.x * kTP >= p) return;
   const bool tip[2] = {(op.flags & OP_TIP1) != 0, (op.flags & OP_TIP2) != 0};
   const void *in[2] = {op.in1, op.in2};
   const T *Pg[2] = {static_cast<const T *>(op.P1), static_cast<const T *>(op.P2)};

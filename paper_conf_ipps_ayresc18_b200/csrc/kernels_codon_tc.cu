@@ -201,7 +201,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
     for (int b = 0; b < 2; ++b)
       if (fl[b] && tid < TM) {
         const int pp = p0 + tid;
-        st_s[((lt & 1) * 2 + b) * TM + tid] = pp < p ? static_cast<const uint8_t *>(in[b])[pp] : (uint8_t)kS61;
+        st_s[((lt & 1) * 2 + b) * TM + tid] = pp < op.p ? static_cast<const uint8_t *>(in[b])[pp] : (uint8_t)kS61;
       }
   };
 
@@ -224,7 +224,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
       for (int u = 0; u < NA; ++u) {
         const int i = tid + u * kThr;
         const int kh = i & 1, rr = (i >> 1) & (TM - 1), kb = i >> 8;
-        fa[u] = (p0 + rr < p) ? __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + (kb * 2 + kh) * 4))
+        fa[u] = (p0 + rr < op.p) ? __ldg(reinterpret_cast<const float4 *>(A + (size_t)rr * TS + (kb * 2 + kh) * 4))
                               : make_float4(0.f, 0.f, 0.f, 0.f);
       }
     }
@@ -343,7 +343,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
     const DevOp &op = ops[f / ntiles];
     const int p0 = (f % ntiles) * TM;
     const int pp = p0 + r;
-    const bool valid = pp < p;
+    const bool valid = pp < op.p;
     float d[32];
 #pragma unroll
     for (int half = 0; half < 2; ++half) {
@@ -387,7 +387,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
 #pragma unroll
         for (int u = 0; u < TM * 16 / kThr; ++u) {
           const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
-          if (p0 + row < p)
+          if (p0 + row < op.p)
             *reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
         }
       }
@@ -443,7 +443,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
 #pragma unroll
             for (int u = 0; u < TM * 16 / kThr; ++u) {
               const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
-              if (p0 + row < p)
+              if (p0 + row < op.p)
                 *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *slot(cat, row, ch);
             }
         } else {
@@ -453,7 +453,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
 #pragma unroll
             for (int u = 0; u < TM * 16 / kThr; ++u) {  // all loads first
               const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
-              v[u] = (p0 + row < p)
+              v[u] = (p0 + row < op.p)
                          ? *reinterpret_cast<const float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4)
                          : make_float4(0.f, 0.f, 0.f, 0.f);
             }
@@ -461,7 +461,7 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
             for (int u = 0; u < TM * 16 / kThr; ++u) {
               const int i = tid + u * kThr, row = i >> 4, ch = i & 15;
               const float sc = mx[row];
-              if (p0 + row < p && sc != 1.f)
+              if (p0 + row < op.p && sc != 1.f)
                 *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) =
                     make_float4(v[u].x * sc, v[u].y * sc, v[u].z * sc, v[u].w * sc);
             }

@@ -215,7 +215,8 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
   const uint8_t *__restrict__ S2g = static_cast<const uint8_t *>(op.in2);
   T *__restrict__ out = static_cast<T *>(op.out);
   const bool scale_w = op.scale_out != nullptr;
-  const unsigned nitems = (unsigned)p * C;
+  const unsigned nitems = (unsigned)op.p * C;  // this operation's pattern range
+  (void)p;
 
   pdl_wait();  // everything above overlaps the previous level set
   pdl_launch();
@@ -333,6 +334,10 @@ __device__ inline void issue_chunk(const DevOp *ops, int oi, int chunk, BulkStag
                                    uint64_t *bar) {
   using S = BulkStage<T, C>;
   const DevOp &op = ops[oi];
+  if ((long long)chunk * kChunkItems >= (long long)op.p * C) {  // beyond this op's pattern range
+    mbar_expect_tx(bar, 0u);
+    return;
+  }
   const bool t1 = op.flags & OP_TIP1, t2 = op.flags & OP_TIP2;
   const bool cum = op.scale_out != nullptr;
   const bool e1 = cum && !t1 && op.cum1 != nullptr, e2 = cum && !t2 && op.cum2 != nullptr;
@@ -498,7 +503,7 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
 
   // ------------------------------------------------------------------ consumers
   const int cat = threadIdx.x % C;
-  const unsigned nitems = (unsigned)p * C;
+  (void)p;
   const int op_lo = lo / nchunks, op_hi = (hi - 1) / nchunks;
   int i = 0;
   for (int oi = op_lo; oi <= op_hi; ++oi) {
@@ -506,6 +511,7 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
     const int c1 = (oi == op_hi) ? (hi - 1) % nchunks + 1 : nchunks;
     consumer_sync();  // previous op's tables no longer in use
     const DevOp op = ops[oi];
+    const unsigned nitems = (unsigned)op.p * C;  // this operation's pattern range
     load_ptables_consumers<T, C>(sP, op);
     T P1[16], P2[16];
 #pragma unroll

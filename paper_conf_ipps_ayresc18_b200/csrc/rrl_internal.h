@@ -26,7 +26,7 @@ struct DevOp {
   const int32_t *cum1;      // child 1 cumulative exponent (cumulative mode) or null
   const int32_t *cum2;      // child 2
   int32_t flags;            // bit0: child1 is tip states, bit1: child2 is tip states
-  int32_t pad;
+  int32_t p;                // patterns of this operation (pointers are pre-offset to its range)
 };
 static_assert(sizeof(DevOp) == 80, "DevOp layout");
 

@@ -38,7 +38,7 @@ class TreeLikelihood:
     def __init__(self, n: int, p: int, s: int, c: int, precision: int = 32, device: int = 0,
                  cumulative_scaling: bool = True, cuda_graph: bool = False,
                  buffer_count: int | None = None, stream_ptr: int | None = None,
-                 codon_simt: bool = False):
+                 codon_simt: bool = False, partitions: int = 1):
         self.n, self.p, self.s, self.c, self.precision = n, p, s, c, precision
         self.cumulative = cumulative_scaling
         nbuf = buffer_count if buffer_count is not None else 2 * n - 1
@@ -47,8 +47,10 @@ class TreeLikelihood:
                 (R.FLAG_CUDA_GRAPH if cuda_graph else 0) | (R.FLAG_CODON_SIMT if codon_simt else 0)
         self.nbuf = nbuf
         self.n_scale = n_scale
-        self.inst = R.rrl_create_instance(n, nbuf, s, p, c, 2 * n - 1, 1, n_scale, device,
-                                          precision, flags)
+        self.partitions = partitions
+        self.ranges = None
+        self.inst = R.rrl_create_instance(n, nbuf, s, p, c, partitions * (2 * n - 1), partitions, n_scale,
+                                          device, precision, flags)
         if stream_ptr is not None:
             R.rrl_set_stream(self.inst, stream_ptr)
         self.sched = None
@@ -68,6 +70,22 @@ class TreeLikelihood:
         """Convenience for any object with name/pi/kappa/omega/exch attributes."""
         return self.set_model(mp.name, mp.pi, rates, cat_weights, getattr(mp, "kappa", 1.0),
                               getattr(mp, "omega", 1.0), getattr(mp, "exch", None))
+
+    def set_partition_model(self, k: int, mp, rates, cat_weights):
+        """Model of partition k (independent parameters per data
+        subset): eigensystem, frequencies, category weights and rates in slot k."""
+        prm = model_param_vector(mp.name, getattr(mp, "kappa", 1.0), getattr(mp, "omega", 1.0),
+                                 getattr(mp, "exch", None))
+        _, V, Vi, lam = R.rrl_model_eigensystem(mp.name, mp.pi, prm)
+        R.rrl_set_eigen_decomposition(self.inst, k, V, Vi, lam)
+        R.rrl_set_state_frequencies(self.inst, k, mp.pi)
+        R.rrl_set_category_rates_idx(self.inst, k, rates)
+        R.rrl_set_category_weights(self.inst, k, cat_weights)
+
+    def set_partition_ranges(self, ranges):
+        """[(begin, end)] per partition; begins multiples of RRL_PATTERN_RANGE_ALIGN."""
+        assert len(ranges) == self.partitions
+        self.ranges = [(int(b), int(e)) for b, e in ranges]
 
     def set_tips(self, tips_u8: np.ndarray):
         R.rrl_set_tip_states_u8(self.inst, 0, tips_u8)
@@ -92,13 +110,38 @@ class TreeLikelihood:
         self.sched = sch
         self.ops = ops
         self.offsets = sch["set_offsets"]
+        self._pops = None
         return sch
 
     # ---------------------------------------------------------------- pass
+    def _partitioned_ops(self):
+        """Every level set of every partition in ONE set: partition k's copy of
+        an op uses matrices k*(2n-1)+node and its own pattern range."""
+        N = 2 * self.n - 1
+        ops, ranges, offs = [], [], [0]
+        for a, b in zip(self.offsets[:-1], self.offsets[1:]):
+            for k, (pb, pe) in enumerate(self.ranges):
+                o = self.ops[a:b].copy()
+                o["matrix1"] += k * N
+                o["matrix2"] += k * N
+                ops.append(o)
+                ranges += [(pb, pe)] * (b - a)
+            offs.append(offs[-1] + (b - a) * self.partitions)
+        return np.concatenate(ops), np.array(ranges, np.int32), np.array(offs, np.int32)
+
     def update(self):
         """K1 + all level-set launches (+ K5 when not cumulative)."""
-        R.rrl_update_transition_matrices(self.inst, 0, self.matrix_idx, self.t)
-        R.rrl_update_partials(self.inst, self.ops, self.offsets)
+        if self.partitions > 1:
+            N = 2 * self.n - 1
+            for k in range(self.partitions):
+                R.rrl_update_transition_matrices(self.inst, k, self.matrix_idx + k * N, self.t)
+            if getattr(self, "_pops", None) is None or self._pops_key is not self.ops:
+                self._pops = self._partitioned_ops()
+                self._pops_key = self.ops
+            R.rrl_update_partials_ranged(self.inst, self._pops[0], self._pops[1], self._pops[2])
+        else:
+            R.rrl_update_transition_matrices(self.inst, 0, self.matrix_idx, self.t)
+            R.rrl_update_partials(self.inst, self.ops, self.offsets)
         if not self.cumulative:
             cum = self.n_scale - 1
             R.rrl_reset_scale_factors(self.inst, cum)
@@ -115,6 +158,12 @@ class TreeLikelihood:
     def root_loglik_device(self, d_out_ptr: int):
         R.rrl_calculate_root_log_likelihoods_device(self.inst, self.root_buffer, 0, 0,
                                                     self.cumulative_idx, d_out_ptr)
+
+    def partition_logliks(self) -> list[float]:
+        """Root log-likelihood of each partition (its model slot, its range)."""
+        return [R.rrl_calculate_root_log_likelihoods_range(self.inst, self.root_buffer, k, k,
+                                                           self.cumulative_idx, b, e)
+                for k, (b, e) in enumerate(self.ranges)]
 
     def loglik(self) -> float:
         self.update()

@@ -40,6 +40,7 @@ SCHED_SEQUENTIAL = 1
 SCHED_LEVEL = 2
 SCHED_REROOT = 3
 SCHED_REUSE_BUFFERS = 0x100
+PATTERN_RANGE_ALIGN = 512
 SCHED_MODES = {"sequential": SCHED_SEQUENTIAL, "level": SCHED_LEVEL, "reroot": SCHED_REROOT}
 
 OP_DTYPE = np.dtype([("dest", "<i4"), ("dest_scale_write", "<i4"), ("dest_scale_read", "<i4"),
@@ -99,6 +100,9 @@ _SIGS = {
     "rrl_reroot_edge_table": (_I, [_I, _P, _P, _P, _P]),
     "rrl_model_eigensystem": (_I, [C.c_char_p, _I, _P, _P, _I, _P, _P, _P, _P]),
     "rrl_schedule_partial": (_I, [_I, _P, _P, _I, _P, _P, _P, _P]),
+    "rrl_set_category_rates_idx": (_I, [_I, _I, _P]),
+    "rrl_update_partials_ranged": (_I, [_I, _P, _P, _I, _P, _I]),
+    "rrl_calculate_root_log_likelihoods_range": (_I, [_I] * 7 + [_P]),
     "rrl_reroot_exhaustive": (_I, [_I, _P, _P, _P, _P]),
 }
 for _name, (_res, _args) in _SIGS.items():
@@ -367,3 +371,28 @@ def rrl_reroot_exhaustive(tip_count, parent, blen=None):
     _chk(_lib.rrl_reroot_exhaustive(tip_count, _ptr(par), _ptr(bl), _ptr(key), _ptr(sets)),
          "rrl_reroot_exhaustive")
     return int(key[0]), int(sets[0])
+
+
+def rrl_set_category_rates_idx(inst, idx, r):
+    a = _c(r, np.float64)
+    return _chk(_lib.rrl_set_category_rates_idx(inst, idx, _ptr(a)), "rrl_set_category_rates_idx")
+
+
+def rrl_update_partials_ranged(inst, ops, pattern_ranges, set_offsets=None):
+    o = as_ops(ops)
+    rg = _c(pattern_ranges, np.int32).reshape(-1)
+    if set_offsets is None:
+        return _chk(_lib.rrl_update_partials_ranged(inst, _ptr(o), _ptr(rg), o.shape[0], None, 0),
+                    "rrl_update_partials_ranged")
+    so = _c(set_offsets, np.int32)
+    return _chk(_lib.rrl_update_partials_ranged(inst, _ptr(o), _ptr(rg), o.shape[0], _ptr(so), so.shape[0] - 1),
+                "rrl_update_partials_ranged")
+
+
+def rrl_calculate_root_log_likelihoods_range(inst, root_buffer, cat_weights_idx, freqs_idx, cumulative_idx,
+                                             pattern_begin, pattern_end) -> float:
+    out = np.zeros(1, dtype=np.float64)
+    _chk(_lib.rrl_calculate_root_log_likelihoods_range(inst, root_buffer, cat_weights_idx, freqs_idx,
+                                                       cumulative_idx, pattern_begin, pattern_end, _ptr(out)),
+         "rrl_calculate_root_log_likelihoods_range")
+    return float(out[0])

@@ -478,3 +478,42 @@ def test_dest_scale_read_reuses_factors(kind, p, model, precision):
         np.testing.assert_array_equal(tl.partials(v), L)
     assert tl.root_loglik() == first
     tl.close()
+
+
+# ------------------------------------------------------------------ pattern partitions (NEXT-3)
+@pytest.mark.parametrize("precision,s_model", [(64, "gtr"), (32, "gtr"), (32, "gy94"), (64, "gy94")])
+def test_pattern_partitions_one_launch_per_set(precision, s_model):
+    """PAPER.md:75-79 §IV-A: partitions with independent models computed
+    concurrently by the multi-operation kernel -- every level set of all
+    partitions is ONE launch; each partition matches the oracle run on its
+    own columns with its own model."""
+    from paper_conf_ipps_ayresc18_b200 import TreeLikelihood, rrl as R
+    from workloads import random_model, discrete_gamma_rates
+    codon = s_model == "gy94"
+    p = 1200 if codon else 2600
+    ranges = [(0, 512), (512, 1024), (1024, p)] if codon else [(0, 1024), (1024, 2048), (2048, p)]
+    w = make_workload(tree_kind="random", n=30, p=p, model=s_model, c=4, seed=41, missing_frac=0.05)
+    rng = np.random.default_rng(5)
+    names = ["gy94"] * 3 if codon else ["gtr", "hky", "gtr"]
+    models = [random_model(nm, rng) for nm in names]
+    rates = [discrete_gamma_rates(a, 4) for a in (0.3, 0.9, 1.7)]
+    cw = np.full(4, 0.25)
+    tl = TreeLikelihood(w.n, p, w.s, 4, precision=precision, partitions=3)
+    for k in range(3):
+        tl.set_partition_model(k, models[k], rates[k], cw)
+    tl.set_partition_ranges(ranges)
+    tl.set_tips(w.tips)
+    tl.set_tree(w.tree.parent, w.tree.blen, "reroot")
+    R.rrl_reset_profile(tl.inst)
+    tl.update()
+    prof = R.rrl_get_profile(tl.inst)
+    assert prof["partials_launches"] == tl.sched["set_count"]   # not 3x
+    got = tl.partition_logliks()
+    for k, (b, e) in enumerate(ranges):
+        sub = make_workload(tree_kind="random", n=30, p=1, model=s_model, c=4, seed=41,
+                            model_params=models[k], alpha=1.0)
+        sub.rates = rates[k]
+        sub.tips = np.ascontiguousarray(w.tips[:, b:e])
+        sub.pattern_weights = np.ones(e - b)
+        assert rel(got[k], oracle_run(sub).lnl) <= LNL_TOL[precision], k
+    tl.close()
