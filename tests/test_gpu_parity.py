@@ -481,7 +481,8 @@ def test_dest_scale_read_reuses_factors(kind, p, model, precision):
 
 
 # ------------------------------------------------------------------ pattern partitions (NEXT-3)
-@pytest.mark.parametrize("precision,s_model", [(64, "gtr"), (32, "gtr"), (32, "gy94"), (64, "gy94")])
+@pytest.mark.parametrize("precision,s_model", [(64, "gtr"), (32, "gtr"), (32, "gy94"), (64, "gy94"),
+                                               (32, "gtr_bulk"), (64, "gtr_bulk")])
 def test_pattern_partitions_one_launch_per_set(precision, s_model):
     """PAPER.md:75-79 §IV-A: partitions with independent models computed
     concurrently by the multi-operation kernel -- every level set of all
@@ -490,8 +491,11 @@ def test_pattern_partitions_one_launch_per_set(precision, s_model):
     from paper_conf_ipps_ayresc18_b200 import TreeLikelihood, rrl as R
     from workloads import random_model, discrete_gamma_rates
     codon = s_model == "gy94"
-    p = 1200 if codon else 2600
-    ranges = [(0, 512), (512, 1024), (1024, p)] if codon else [(0, 1024), (1024, 2048), (2048, p)]
+    bulk = s_model == "gtr_bulk"           # >= 64 K items per op: the bulk-copy kernel
+    s_model = "gtr" if bulk else s_model
+    p = 1200 if codon else (40_000 if bulk else 2600)
+    ranges = ([(0, 512), (512, 1024), (1024, p)] if codon else
+              [(0, 20_480), (20_480, 33_280), (33_280, p)] if bulk else [(0, 1024), (1024, 2048), (2048, p)])
     w = make_workload(tree_kind="random", n=30, p=p, model=s_model, c=4, seed=41, missing_frac=0.05)
     rng = np.random.default_rng(5)
     names = ["gy94"] * 3 if codon else ["gtr", "hky", "gtr"]
