@@ -382,7 +382,9 @@ def main():
             # contraction; algorithmic bytes count 61 states (the 64-wide
             # padding is overhead).  Tensor work for context.
             res["roofline"]["tensor_tflops"] = fl / (part_ms * 1e-3) / 1e12
-            res["roofline"]["kernel"] = "k_partials_codon_tc (tcgen05 kind::tf32, 3xTF32)"
+            res["roofline"]["kernel"] = ("k_partials_codon_tc5 (TMA-fed tcgen05 kind::tf32, 3xTF32)"
+                                         if os.environ.get("RRL_CODON_TC5", "1") != "0" else
+                                         "k_partials_codon_tc (tcgen05 kind::tf32, 3xTF32)")
         if s == 61 and precision == 64:
             # SIMT fp64 codon kernel: bound by FP64 FMA issue, not HBM
             peak_tf = 148 * 64 * 2 * 1.965e9 / 1e12

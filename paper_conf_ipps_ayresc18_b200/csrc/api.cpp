@@ -7,10 +7,13 @@
 // device descriptors (DevOp) once per distinct operation list, then issues
 // ONE kernel launch per concurrent operation set, optionally
 // captured into a CUDA graph and replayed.
+#include <cuda.h>  // CUtensorMap (encoded through the runtime's driver entry point)
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <string>
@@ -86,6 +89,10 @@ struct Instance {
   std::vector<EvPair> events;
   std::vector<cudaEvent_t> ev_pool;
   rrl_profile prof{};
+
+  // TMA descriptors of the internal-partials and matrix slabs (61-state fp32, K3-TC5)
+  CUtensorMap tmap_partials{}, tmap_P{};
+  bool tmaps_ok = false;
 };
 
 std::mutex g_mu;
@@ -342,6 +349,31 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
   CKC(cudaMalloc(&I->d_out, sizeof(double)));
   CKC(cudaMalloc(&I->d_count, sizeof(unsigned)));
   CKC(cudaMemset(I->d_count, 0, sizeof(unsigned)));
+  if (state_count == 61 && precision == 32 && n_int > 0) {
+    // 4-D maps, innermost first: internal partials {64 states, p_pad, c, buffer},
+    // matrices {64 child states, 64 parent states, c, matrix}; boxes of 32 states
+    // (one 128-byte swizzle row) x 128 patterns / 64 parent states.
+    const char *env = std::getenv("RRL_CODON_TC5");
+    PFN_cuTensorMapEncodeTiled_v12000 enc = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (!(env && env[0] == '0') &&
+        cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void **)&enc, cudaEnableDefault, &q) == cudaSuccess &&
+        enc != nullptr && n_int <= 0x7fffffff) {
+      const cuuint64_t gA[4] = {64, (cuuint64_t)I->p_pad, (cuuint64_t)I->c, (cuuint64_t)n_int};
+      const cuuint64_t sA[3] = {256, (cuuint64_t)I->p_pad * 256, (cuuint64_t)I->buf_bytes};
+      const cuuint32_t bA[4] = {32, 128, 1, 1}, es[4] = {1, 1, 1, 1};
+      const cuuint64_t gP[4] = {64, 64, (cuuint64_t)I->c, (cuuint64_t)matrix_count};
+      const cuuint64_t sP[3] = {256, 64 * 256, (cuuint64_t)I->c * 64 * 256};
+      const cuuint32_t bP[4] = {32, 64, 1, 1};
+      const CUresult r1 = enc(&I->tmap_partials, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, I->d_partials, gA, sA, bA, es,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      const CUresult r2 = enc(&I->tmap_P, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, I->d_P, gP, sP, bP, es,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      I->tmaps_ok = (r1 == CUDA_SUCCESS && r2 == CUDA_SUCCESS);
+    }
+  }
   CKC(cudaMallocHost(&I->h_out, sizeof(double)));
   {
     std::vector<double> ones(I->p_pad, 1.0), r((size_t)category_count * eigen_count, 1.0),
@@ -708,6 +740,11 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       child(o.child1, &d.in1, &d.cum1, OP_TIP1);
       child(o.child2, &d.in2, &d.cum2, OP_TIP2);
       d.out = buffer_ptr(I, o.dest);
+      d.buf1 = (o.child1 >= I->n_tips) ? o.child1 - I->n_tips : -1;
+      d.buf2 = (o.child2 >= I->n_tips) ? o.child2 - I->n_tips : -1;
+      d.mat1 = o.matrix1;
+      d.mat2 = o.matrix2;
+      d.pat0 = ranges ? ranges[2 * i] : 0;
       d.P1 = I->d_P + (size_t)o.matrix1 * I->mat_elems * I->elt;
       d.P2 = I->d_P + (size_t)o.matrix2 * I->mat_elems * I->elt;
       d.scale_out = o.dest_scale_write >= 0 ? I->d_scale + (size_t)o.dest_scale_write * I->p_pad : nullptr;
@@ -760,7 +797,10 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
                                        I->p_pad, I->stream);
       } else {
         e = (int)cudaErrorNotSupported;
-        if (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))  // tcgen05 path (c <= 4)
+        if (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT) && I->tmaps_ok)  // TMA-fed tcgen05 (c <= 4)
+          e = launch_update_partials_codon_tc5(I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax, I->p_pad,
+                                               &I->tmap_partials, &I->tmap_P, I->stream);
+        if (e == (int)cudaErrorNotSupported && I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))
           e = launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, pmax, I->p_pad, I->stream);
         if (e == (int)cudaErrorNotSupported)
           e = launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax,

@@ -1,0 +1,432 @@
+// K3-TC5: 61-state codon updatePartials, TMA-fed tcgen05 pipeline (fp32, c <= 4).
+//
+// Eq. (1) (§II-A) for s = 61: per operation, category c and
+// 128-pattern tile, D_b = A_b . P_b^T for both children (A_b: [128 x 64]
+// child partials, P_b: [64 x 64] transition matrix, K-major = its natural
+// row-major layout), out = D_1 .* D_2, rescaled per pattern by the exact
+// power of two of max over (c, z).
+//
+// Pipeline of phases (tile, category, child) through four warp roles, joined
+// only by mbarriers (no block-wide barrier in steady state):
+//  * producer (warp 12, one lane): TMA (cp.async.bulk.tensor.4d) of the
+//    child tile straight from the [buffer][c][p_pad][64] partials slab and of
+//    the P tile from the [matrix][c][64][64] slab into one of two 96 KB
+//    stages, 128-byte swizzled -- the canonical SWIZZLE_128B K-major UMMA
+//    layout, so the raw fp32 tile IS the tf32 "hi" operand (the tensor core
+//    reads the top 19 bits of each 32-bit element);
+//  * converters (warps 8-11): the tf32 "lo" parts, lo = rn_tf32(x - hi(x)),
+//    elementwise in place of layout (same swizzled offsets), for A and P; a
+//    tip child's A tile is built one-hot (all ones for a missing state) and
+//    needs no lo;
+//  * MMA issuer (warp 13, one lane): per K-step of 8, hi*hi into one of four
+//    main accumulators and hi*lo + lo*hi into a correction accumulator (the
+//    accumulation-precision scheme measured in DESIGN.md), tcgen05.commit to
+//    the stage's `empty` and to `acc_full`;
+//  * epilogue (warps 0-7: TMEM lane quarter w%4, column half w/4): sums the
+//    five accumulators (tcgen05.ld 32x32b.x16), releases `acc_empty`, parks
+//    child 1 in shared memory, forms the product with child 2, parks it in
+//    TMEM until the tile's last category, then scales by 2^-e and writes every
+//    category once, coalesced, through a swizzled staging tile.
+// Compared with K3-TC (kernels_codon_tc.cu) the SM no longer moves the child
+// tile through registers: per phase it only writes the lo halves.
+#include <cuda.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "rrl_internal.h"
+
+namespace rrl {
+namespace {
+
+constexpr int TM = 128;  // patterns per tile = MMA M = TMEM lanes
+constexpr int TS = 64;   // padded states: MMA N and K
+constexpr int kS61 = 61;
+constexpr int kEpiThr = 256;                 // warps 0-7
+constexpr int kConvThr = 128;                // warps 8-11
+constexpr int kProdWarp = 12, kMmaWarp = 13;
+constexpr int kThr = 14 * 32;
+// one stage: A hi (2 x 16 KB halves k 0-31 / 32-63), A lo, P hi (2 x 8 KB), P lo
+constexpr int ST_AHI = 0, ST_ALO = 32768, ST_BHI = 65536, ST_BLO = 81920, ST_BYTES = 98304;
+constexpr int SMEM_S1 = 2 * ST_BYTES;                  // epilogue staging tile (32 KB)
+constexpr int SMEM_MX = SMEM_S1 + TM * TS * 4;         // row maxima / scale [2][128]
+constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 8 mbarriers
+constexpr int SMEM_TMEM = SMEM_BAR + 8 * 8;
+constexpr int SMEM_TOTAL = SMEM_TMEM + 16;
+constexpr int kTmemCols = 512;    // 4 main + 1 correction accumulator (5 x 64) ...
+constexpr int kProdCol = 5 * TS;  // ... + parked products of categories 0..C-2
+
+__device__ inline uint32_t sa(const void *p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
+__device__ inline uint64_t desc_sw128(uint32_t saddr) {  // K-major, 128-byte swizzle, 8-row atoms of 1 KB
+  return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
+         ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(TS >> 3) << 17) |
+                            ((uint32_t)(TM >> 4) << 24);  // kind::tf32, D f32, K-major A/B, N 64, M 128
+
+__device__ inline void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t acc) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
+      "l"(a), "l"(b), "r"(kIdesc), "r"(acc));
+}
+__device__ inline void commit(uint64_t *bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(sa(bar))
+               : "memory");
+}
+__device__ inline void bar_init(uint64_t *bar, unsigned n) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(sa(bar)), "r"(n));
+}
+__device__ inline void bar_arrive(uint64_t *bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(sa(bar)) : "memory");
+}
+__device__ inline void bar_expect(uint64_t *bar, unsigned bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(sa(bar)), "r"(bytes) : "memory");
+}
+__device__ inline void bar_wait(uint64_t *bar, uint32_t parity) {
+  asm volatile(
+      "{\n.reg .pred P1;\nW_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra W_%=;\n}\n" ::"r"(sa(bar)),
+      "r"(parity)
+      : "memory");
+}
+__device__ inline void tma4(uint32_t dst, const void *tmap, int x, int y, int z, int w, uint64_t *bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3, %4, %5}], [%6];" ::"r"(
+          dst),
+      "l"(tmap), "r"(x), "r"(y), "r"(z), "r"(w), "r"(sa(bar))
+      : "memory");
+}
+__device__ inline void tmem_ld16(uint32_t taddr, float (&v)[16]) {
+  uint32_t r[16];
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+        "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
+      : "r"(taddr));
+#pragma unroll
+  for (int i = 0; i < 16; ++i) v[i] = __uint_as_float(r[i]);
+}
+__device__ inline void tmem_st16(uint32_t taddr, const float *v) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(taddr),
+      "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])), "r"(__float_as_uint(v[3])),
+      "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])), "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])),
+      "r"(__float_as_uint(v[8])), "r"(__float_as_uint(v[9])), "r"(__float_as_uint(v[10])), "r"(__float_as_uint(v[11])),
+      "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])), "r"(__float_as_uint(v[14])), "r"(__float_as_uint(v[15]))
+      : "memory");
+}
+__device__ inline void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+__device__ inline void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
+__device__ inline void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ inline void fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+__device__ inline void named_sync(int id, int n) { asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(n) : "memory"); }
+
+__device__ inline float lo_tf32(float x) {  // rn_tf32(x - trunc_tf32(x))
+  const float hi = __uint_as_float(__float_as_uint(x) & 0xffffe000u);
+  return __uint_as_float((__float_as_uint(x - hi) + 0x1000u) & 0xffffe000u);
+}
+__device__ inline int frexp_e(float m) {
+  const unsigned b = __float_as_uint(m);
+  const int eb = (int)((b >> 23) & 0xffu);
+  if (eb != 0 && eb != 0xff) return eb - 126;
+  if (m == 0.f) return 0;
+  int e;
+  frexpf(m, &e);
+  return e;
+}
+
+template <int C>
+__global__ void __launch_bounds__(kThr, 1)
+k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p_pad,
+                     const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmP) {
+  static_assert(kProdCol + (C - 1) * TS <= kTmemCols, "parked products must fit TMEM");
+  extern __shared__ __align__(1024) unsigned char sm[];
+  uint64_t *tma_full = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);  // [2]
+  uint64_t *conv_full = tma_full + 2;                                 // [2]
+  uint64_t *empty = tma_full + 4;                                     // [2]
+  uint64_t *acc_full = tma_full + 6;
+  uint64_t *acc_empty = tma_full + 7;
+  uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(sm + SMEM_TMEM);
+  float *S1 = reinterpret_cast<float *>(sm + SMEM_S1);
+  float *mx = reinterpret_cast<float *>(sm + SMEM_MX);
+  const uint32_t sbase = sa(sm);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if ((sbase & 1023u) != 0u) __trap();  // swizzled stages need 1 KB alignment
+
+  if (warp == 0) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(sa(tmem_slot)),
+                 "r"(kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  if (tid == kProdWarp * 32) {
+    for (int s = 0; s < 2; ++s) {
+      bar_init(&tma_full[s], 1);
+      bar_init(&conv_full[s], kConvThr / 32);
+      bar_init(&empty[s], 1);
+    }
+    bar_init(acc_full, 1);
+    bar_init(acc_empty, kEpiThr / 32);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmP) : "memory");
+  }
+  fence_before();
+  __syncthreads();
+  fence_after();
+  const uint32_t tmem = *tmem_slot;
+  asm volatile("griddepcontrol.wait;" ::: "memory");  // everything above overlaps the previous level set
+  asm volatile("griddepcontrol.launch_dependents;" :::);
+
+  const int my_tiles = total > (int)blockIdx.x ? (total - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
+  const int nphase = my_tiles * C * 2;  // (tile, category, child)
+
+  if (warp == kProdWarp) {
+    // ================================================================ TMA producer
+    if (lane == 0) {
+      for (int g = 0; g < nphase; ++g) {
+        const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1, s = g & 1;
+        const int f = blockIdx.x + lt * gridDim.x;
+        const DevOp &op = ops[f / ntiles];
+        const int p0 = (f % ntiles) * TM;
+        const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+        const int buf = b == 0 ? op.buf1 : op.buf2, mat = b == 0 ? op.mat1 : op.mat2;
+        bar_wait(&empty[s], ((uint32_t)(g >> 1) & 1u) ^ 1u);  // MMAs of phase g-2 are done
+        const uint32_t st = sbase + s * ST_BYTES;
+        bar_expect(&tma_full[s], (tip ? 0u : 32768u) + 16384u);
+        if (!tip) {
+          tma4(st + ST_AHI, &tmA, 0, op.pat0 + p0, c, buf, &tma_full[s]);
+          tma4(st + ST_AHI + 16384, &tmA, 32, op.pat0 + p0, c, buf, &tma_full[s]);
+        }
+        tma4(st + ST_BHI, &tmP, 0, 0, c, mat, &tma_full[s]);
+        tma4(st + ST_BHI + 8192, &tmP, 32, 0, c, mat, &tma_full[s]);
+      }
+    }
+  } else if (warp == kMmaWarp) {
+    // ================================================================ MMA issuer
+    if (lane == 0) {
+      for (int g = 0; g < nphase; ++g) {
+        const int lt = g / (2 * C), b = g & 1, s = g & 1;
+        const int f = blockIdx.x + lt * gridDim.x;
+        const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+        bar_wait(&conv_full[s], (uint32_t)(g >> 1) & 1u);
+        bar_wait(acc_empty, (uint32_t)(g & 1) ^ 1u);  // epilogue g-1 drained the accumulators
+        fence_after();
+        const uint32_t st = sbase + s * ST_BYTES;
+#pragma unroll
+        for (int kk = 0; kk < TS / 8; ++kk) {
+          const int h = kk >> 2, kin = kk & 3;
+          const uint64_t ah = desc_sw128(st + ST_AHI + h * 16384 + kin * 32);
+          const uint64_t al = desc_sw128(st + ST_ALO + h * 16384 + kin * 32);
+          const uint64_t bh = desc_sw128(st + ST_BHI + h * 8192 + kin * 32);
+          const uint64_t bl = desc_sw128(st + ST_BLO + h * 8192 + kin * 32);
+          const uint32_t dmain = tmem + (uint32_t)((kk >> 1) * TS), dcorr = tmem + (uint32_t)(4 * TS);
+          mma_tf32(dmain, ah, bh, (kk & 1) ? 1u : 0u);
+          mma_tf32(dcorr, ah, bl, kk > 0 ? 1u : 0u);
+          if (!tip) mma_tf32(dcorr, al, bh, 1u);
+        }
+        commit(&empty[s]);  // stage free once these MMAs completed
+        commit(acc_full);   // accumulators ready for the epilogue
+      }
+    }
+  } else if (warp >= kEpiThr / 32) {
+    // ================================================================ converters
+    const int ct = tid - kEpiThr;
+    for (int g = 0; g < nphase; ++g) {
+      const int lt = g / (2 * C), b = g & 1, s = g & 1;
+      const int f = blockIdx.x + lt * gridDim.x;
+      const DevOp &op = ops[f / ntiles];
+      const int p0 = (f % ntiles) * TM;
+      const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+      unsigned char *st = sm + s * ST_BYTES;
+      bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
+      if (!tip) {
+#pragma unroll 4
+        for (int i = ct; i < TM * 16; i += kConvThr) {  // lo of every 16-byte chunk, same swizzled offset
+          const float4 v = *reinterpret_cast<const float4 *>(st + ST_AHI + i * 16);
+          *reinterpret_cast<float4 *>(st + ST_ALO + i * 16) =
+              make_float4(lo_tf32(v.x), lo_tf32(v.y), lo_tf32(v.z), lo_tf32(v.w));
+        }
+      } else {
+        const uint8_t *states = static_cast<const uint8_t *>(b == 0 ? op.in1 : op.in2);  // range-offset
+#pragma unroll 4
+        for (int i = ct; i < TM * 16; i += kConvThr) {  // one-hot rows in the swizzled layout
+          const int h = i >> 10, r = (i >> 3) & (TM - 1), j8 = (i & 7) ^ (r & 7);
+          const unsigned sv = (p0 + r < op.p) ? (unsigned)states[p0 + r] : (unsigned)kS61;
+          float v[4];
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const unsigned k = (unsigned)(h * 32 + j8 * 4 + q);
+            v[q] = (sv < (unsigned)kS61) ? (k == sv ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
+          }
+          *reinterpret_cast<float4 *>(st + ST_AHI + i * 16) = make_float4(v[0], v[1], v[2], v[3]);
+        }
+      }
+#pragma unroll 2
+      for (int i = ct; i < TS * 16; i += kConvThr) {
+        const float4 v = *reinterpret_cast<const float4 *>(st + ST_BHI + i * 16);
+        *reinterpret_cast<float4 *>(st + ST_BLO + i * 16) =
+            make_float4(lo_tf32(v.x), lo_tf32(v.y), lo_tf32(v.z), lo_tf32(v.w));
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
+      __syncwarp();
+      if (lane == 0) bar_arrive(&conv_full[s]);
+    }
+  } else {
+    // ================================================================ epilogue
+    const int h = warp >> 2;               // column half
+    const int r = (warp & 3) * 32 + lane;  // TMEM lane = pattern row of the tile
+    const uint32_t tl = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)(h * 32);
+    auto s1 = [&](int row, int k) -> float4 * {  // 16 x 16-byte chunks per row, chunk k at k ^ (row & 15)
+      return reinterpret_cast<float4 *>(S1 + row * TS + 4 * (k ^ (row & 15)));
+    };
+    float m = 0.f;  // child 1 of the current category waits in this thread's own S1 half-row
+    for (int g = 0; g < nphase; ++g) {
+      const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
+      const int f = blockIdx.x + lt * gridDim.x;
+      const DevOp &op = ops[f / ntiles];
+      const int p0 = (f % ntiles) * TM;
+      const int pp = p0 + r;
+      const bool valid = pp < op.p;
+      bar_wait(acc_full, (uint32_t)g & 1u);
+      fence_after();
+      float dv[32];
+#pragma unroll
+      for (int q = 0; q < 2; ++q) {
+        float a0[16], a1[16], a2[16], a3[16], cc[16];
+        tmem_ld16(tl + 0 * TS + q * 16, a0);
+        tmem_ld16(tl + 1 * TS + q * 16, a1);
+        tmem_ld16(tl + 2 * TS + q * 16, a2);
+        tmem_ld16(tl + 3 * TS + q * 16, a3);
+        tmem_ld16(tl + 4 * TS + q * 16, cc);
+        tmem_wait_ld();
+#pragma unroll
+        for (int i = 0; i < 16; ++i) dv[q * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
+      }
+      fence_before();
+      __syncwarp();
+      if (lane == 0) bar_arrive(acc_empty);  // the MMAs of phase g+1 may overwrite them
+      if (b == 0) {
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          *s1(r, h * 8 + k) = make_float4(dv[4 * k], dv[4 * k + 1], dv[4 * k + 2], dv[4 * k + 3]);
+        continue;
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const float4 w = *s1(r, h * 8 + k);
+        dv[4 * k] *= w.x; dv[4 * k + 1] *= w.y; dv[4 * k + 2] *= w.z; dv[4 * k + 3] *= w.w;
+        m = fmaxf(m, fmaxf(fmaxf(dv[4 * k], dv[4 * k + 1]), fmaxf(dv[4 * k + 2], dv[4 * k + 3])));
+      }
+      if (c < C - 1) {  // park the unscaled product until the tile's exponent is known
+        tmem_st16(tl + (uint32_t)(kProdCol + c * TS), dv);
+        tmem_st16(tl + (uint32_t)(kProdCol + c * TS + 16), dv + 16);
+        tmem_wait_st();
+        continue;
+      }
+      // ---- tile done: row exponent from max over (c, z) of both column halves
+      mx[h * TM + r] = m;
+      named_sync(1, kEpiThr);
+      if (h == 0) {
+        const float mm = fmaxf(mx[r], mx[TM + r]);
+        int e = 0;
+        if (op.scale_out != nullptr) {
+          e = frexp_e(mm);
+          if (valid) {
+            int tot = e;
+            if (op.cum1 != nullptr) tot += op.cum1[pp];
+            if (op.cum2 != nullptr) tot += op.cum2[pp];
+            op.scale_out[pp] = tot;
+          }
+        } else if (op.scale_in != nullptr) {
+          e = valid ? op.scale_in[pp] : 0;
+        }
+        mx[r] = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
+      }
+      named_sync(1, kEpiThr);
+      const float sc = mx[r];
+      float *out = static_cast<float *>(op.out);
+      for (int cat = 0; cat < C; ++cat) {
+        float v[32];
+        if (cat < C - 1) {
+          float lo16[16], hi16[16];
+          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), lo16);
+          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), hi16);
+          tmem_wait_ld();
+#pragma unroll
+          for (int i = 0; i < 16; ++i) { v[i] = lo16[i]; v[16 + i] = hi16[i]; }
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = dv[i];
+        }
+        named_sync(1, kEpiThr);  // staging tile free
+#pragma unroll
+        for (int k = 0; k < 8; ++k)
+          *s1(r, h * 8 + k) = make_float4(v[4 * k] * sc, v[4 * k + 1] * sc, v[4 * k + 2] * sc, v[4 * k + 3] * sc);
+        named_sync(1, kEpiThr);
+#pragma unroll
+        for (int u = 0; u < TM * 16 / kEpiThr; ++u) {  // coalesced: a warp writes 2 rows
+          const int i = tid + u * kEpiThr, row = i >> 4, ch = i & 15;
+          if (p0 + row < op.p)
+            *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
+        }
+      }
+      named_sync(1, kEpiThr);  // staging reads done before rows are reused for child 1
+      m = 0.f;
+    }
+  }
+  fence_before();
+  __syncthreads();
+  if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
+}
+
+template <int C>
+int launch_tc5(const DevOp *d_ops, int nops, int p, int p_pad, const CUtensorMap *tA, const CUtensorMap *tP,
+               cudaStream_t st) {
+  static int nsm = 0;
+  if (nsm == 0) {
+    cudaError_t e = cudaFuncSetAttribute(k_partials_codon_tc5<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         SMEM_TOTAL);
+    if (e != cudaSuccess) return (int)e;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+  }
+  const int ntiles = (p + TM - 1) / TM;
+  const long long total = (long long)ntiles * nops;
+  if (total > 0x7fffffffLL) return (int)cudaErrorInvalidValue;
+  const int grid = (int)(total < nsm ? total : nsm);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3(grid);
+  cfg.blockDim = dim3(kThr);
+  cfg.dynamicSmemBytes = SMEM_TOTAL;
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_codon_tc5<C>, d_ops, ntiles, (int)total, p_pad, *tA, *tP);
+}
+
+}  // namespace
+
+int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
+                                     int p_pad, const void *tmap_partials, const void *tmap_P, void *stream) {
+  // every child must live in the tensor-mapped slab (internal buffers) or be tip states
+  for (int i = 0; i < nops; ++i)
+    if ((!(h_ops[i].flags & OP_TIP1) && h_ops[i].buf1 < 0) || (!(h_ops[i].flags & OP_TIP2) && h_ops[i].buf2 < 0))
+      return (int)cudaErrorNotSupported;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const CUtensorMap *tA = static_cast<const CUtensorMap *>(tmap_partials);
+  const CUtensorMap *tP = static_cast<const CUtensorMap *>(tmap_P);
+  switch (c) {
+    case 1: return launch_tc5<1>(d_ops, nops, p, p_pad, tA, tP, st);
+    case 2: return launch_tc5<2>(d_ops, nops, p, p_pad, tA, tP, st);
+    case 4: return launch_tc5<4>(d_ops, nops, p, p_pad, tA, tP, st);
+    default: return (int)cudaErrorNotSupported;
+  }
+}
+
+}  // namespace rrl

@@ -27,8 +27,13 @@ struct DevOp {
   const int32_t *cum2;      // child 2
   int32_t flags;            // bit0: child1 is tip states, bit1: child2 is tip states
   int32_t p;                // patterns of this operation (pointers are pre-offset to its range)
+  // tensor-map coordinates for the TMA-fed codon kernel (K3-TC5)
+  int32_t buf1, buf2;       // child internal-buffer index in the partials slab, -1 if not in it
+  int32_t mat1, mat2;       // transition-matrix indices
+  int32_t pat0;             // first pattern of the range
+  int32_t pad_;
 };
-static_assert(sizeof(DevOp) == 80, "DevOp layout");
+static_assert(sizeof(DevOp) == 104, "DevOp layout");
 
 enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2 };
 
@@ -42,6 +47,12 @@ int launch_update_partials_codon(int prec, int c, const DevOp *d_ops, const DevO
                                  int p, int p_pad, void *stream);
 // tcgen05 (tf32, 3xTF32) codon kernel: fp32, c in {1,2,4,8}; cudaErrorNotSupported otherwise.
 int launch_update_partials_codon_tc(int c, const DevOp *d_ops, int nops, int p, int p_pad, void *stream);
+// TMA-fed tcgen05 codon kernel: A tiles and P tiles arrive by TMA from the
+// partials slab / matrix slab tensor maps (opaque 128-byte CUtensorMap values
+// passed as void*), converter warps derive the tf32 lo parts in shared memory.
+// cudaErrorNotSupported when a child of the set is not in the slab.
+int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
+                                     int p_pad, const void *tmap_partials, const void *tmap_P, void *stream);
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
                                int count, void *d_P, void *stream);
