@@ -15,9 +15,11 @@
 //    layout, so the raw fp32 tile IS the tf32 "hi" operand (the tensor core
 //    reads the top 19 bits of each 32-bit element);
 //  * converters (warps 8-11): the tf32 "lo" parts, lo = rn_tf32(x - hi(x)),
-//    elementwise in place of layout (same swizzled offsets), for A and P; a
-//    tip child's A tile is built one-hot (all ones for a missing state) and
-//    needs no lo;
+//    elementwise in place of layout (same swizzled offsets), for A and P;
+//  * a tip child (uint8 states) is no contraction at all: sum_x P[z][x] [x = obs]
+//    = P[z][obs], so its phase lands only the raw P tile and the epilogue
+//    gathers the column from shared memory (row sums for a missing state) --
+//    no conversion, no MMA, no TMEM traffic;
 //  * MMA issuer (warp 13, one lane): per K-step of 8, hi*hi into one of four
 //    main accumulators and hi*lo + lo*hi into a correction accumulator (the
 //    accumulation-precision scheme measured in DESIGN.md), tcgen05.commit to
@@ -206,12 +208,15 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
   } else if (warp == kMmaWarp) {
     // ================================================================ MMA issuer
     if (lane == 0) {
+      uint32_t ni = 0;  // internal-child phases issued (accumulator barrier parity)
       for (int g = 0; g < nphase; ++g) {
         const int lt = g / (2 * C), b = g & 1, s = g & 1;
         const int f = blockIdx.x + lt * gridDim.x;
         const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
         bar_wait(&conv_full[s], (uint32_t)(g >> 1) & 1u);
-        bar_wait(acc_empty, (uint32_t)(g & 1) ^ 1u);  // epilogue g-1 drained the accumulators
+        if (tip) continue;  // a tip child is a P-column gather in the epilogue: no MMA
+        bar_wait(acc_empty, (ni & 1u) ^ 1u);  // the epilogue drained the previous accumulators
+        ++ni;
         fence_after();
         const uint32_t st = sbase + s * ST_BYTES;
 #pragma unroll
@@ -224,7 +229,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
           const uint32_t dmain = tmem + (uint32_t)((kk >> 1) * TS), dcorr = tmem + (uint32_t)(4 * TS);
           mma_tf32(dmain, ah, bh, (kk & 1) ? 1u : 0u);
           mma_tf32(dcorr, ah, bl, kk > 0 ? 1u : 0u);
-          if (!tip) mma_tf32(dcorr, al, bh, 1u);
+          mma_tf32(dcorr, al, bh, 1u);
         }
         commit(&empty[s]);  // stage free once these MMAs completed
         commit(acc_full);   // accumulators ready for the epilogue
@@ -236,38 +241,22 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     for (int g = 0; g < nphase; ++g) {
       const int lt = g / (2 * C), b = g & 1, s = g & 1;
       const int f = blockIdx.x + lt * gridDim.x;
-      const DevOp &op = ops[f / ntiles];
-      const int p0 = (f % ntiles) * TM;
-      const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+      const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
       unsigned char *st = sm + s * ST_BYTES;
       bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
-      if (!tip) {
+      if (!tip) {  // a tip phase only lands P for the epilogue's gather: nothing to convert
 #pragma unroll 4
         for (int i = ct; i < TM * 16; i += kConvThr) {  // lo of every 16-byte chunk, same swizzled offset
           const float4 v = *reinterpret_cast<const float4 *>(st + ST_AHI + i * 16);
           *reinterpret_cast<float4 *>(st + ST_ALO + i * 16) =
               make_float4(lo_tf32(v.x), lo_tf32(v.y), lo_tf32(v.z), lo_tf32(v.w));
         }
-      } else {
-        const uint8_t *states = static_cast<const uint8_t *>(b == 0 ? op.in1 : op.in2);  // range-offset
-#pragma unroll 4
-        for (int i = ct; i < TM * 16; i += kConvThr) {  // one-hot rows in the swizzled layout
-          const int h = i >> 10, r = (i >> 3) & (TM - 1), j8 = (i & 7) ^ (r & 7);
-          const unsigned sv = (p0 + r < op.p) ? (unsigned)states[p0 + r] : (unsigned)kS61;
-          float v[4];
-#pragma unroll
-          for (int q = 0; q < 4; ++q) {
-            const unsigned k = (unsigned)(h * 32 + j8 * 4 + q);
-            v[q] = (sv < (unsigned)kS61) ? (k == sv ? 1.f : 0.f) : (k < (unsigned)kS61 ? 1.f : 0.f);
-          }
-          *reinterpret_cast<float4 *>(st + ST_AHI + i * 16) = make_float4(v[0], v[1], v[2], v[3]);
-        }
-      }
 #pragma unroll 2
-      for (int i = ct; i < TS * 16; i += kConvThr) {
-        const float4 v = *reinterpret_cast<const float4 *>(st + ST_BHI + i * 16);
-        *reinterpret_cast<float4 *>(st + ST_BLO + i * 16) =
-            make_float4(lo_tf32(v.x), lo_tf32(v.y), lo_tf32(v.z), lo_tf32(v.w));
+        for (int i = ct; i < TS * 16; i += kConvThr) {
+          const float4 v = *reinterpret_cast<const float4 *>(st + ST_BHI + i * 16);
+          *reinterpret_cast<float4 *>(st + ST_BLO + i * 16) =
+              make_float4(lo_tf32(v.x), lo_tf32(v.y), lo_tf32(v.z), lo_tf32(v.w));
+        }
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
       __syncwarp();
@@ -282,6 +271,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       return reinterpret_cast<float4 *>(S1 + row * TS + 4 * (k ^ (row & 15)));
     };
     float m = 0.f;  // child 1 of the current category waits in this thread's own S1 half-row
+    uint32_t ni = 0;  // internal-child phases consumed (accumulator barrier parity)
     for (int g = 0; g < nphase; ++g) {
       const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
       const int f = blockIdx.x + lt * gridDim.x;
@@ -289,24 +279,60 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       const int p0 = (f % ntiles) * TM;
       const int pp = p0 + r;
       const bool valid = pp < op.p;
-      bar_wait(acc_full, (uint32_t)g & 1u);
-      fence_after();
       float dv[32];
+      if (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) {
+        // Tip child: sum_x P[z][x] [x == obs] = P[z][obs], read from the raw fp32 P tile the
+        // producer landed in stage g&1 (swizzled K-major: row z, 16-byte chunk (x&31)/4 at
+        // position chunk ^ (z&7) of half x>>5). A missing state (code >= 61) is the row sum.
+        const int s = g & 1;
+        bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
+        const unsigned char *pt = sm + s * ST_BYTES + ST_BHI;
+        const uint8_t *states = static_cast<const uint8_t *>(b == 0 ? op.in1 : op.in2);  // range-offset
+        const unsigned sv = valid ? (unsigned)states[pp] : 0u;
+        if (sv < (unsigned)kS61) {
+          const unsigned char *base = pt + (sv >> 5) * 8192 + (sv & 3) * 4;
+          const unsigned j = (sv & 31) >> 2;
 #pragma unroll
-      for (int q = 0; q < 2; ++q) {
-        float a0[16], a1[16], a2[16], a3[16], cc[16];
-        tmem_ld16(tl + 0 * TS + q * 16, a0);
-        tmem_ld16(tl + 1 * TS + q * 16, a1);
-        tmem_ld16(tl + 2 * TS + q * 16, a2);
-        tmem_ld16(tl + 3 * TS + q * 16, a3);
-        tmem_ld16(tl + 4 * TS + q * 16, cc);
-        tmem_wait_ld();
+          for (int i = 0; i < 32; ++i) {
+            const int z = h * 32 + i;
+            dv[i] = *reinterpret_cast<const float *>(base + z * 128 + ((j ^ (unsigned)(z & 7)) << 4));
+          }
+        } else {
 #pragma unroll
-        for (int i = 0; i < 16; ++i) dv[q * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
+          for (int i = 0; i < 32; ++i) dv[i] = 0.f;
+#pragma unroll 1
+          for (int x = 0; x < kS61; ++x) {
+            const unsigned char *base = pt + (x >> 5) * 8192 + (x & 3) * 4;
+            const unsigned j = (unsigned)(x & 31) >> 2;
+#pragma unroll
+            for (int i = 0; i < 32; ++i) {
+              const int z = h * 32 + i;
+              dv[i] += *reinterpret_cast<const float *>(base + z * 128 + ((j ^ (unsigned)(z & 7)) << 4));
+            }
+          }
+        }
+        named_sync(1, kEpiThr);  // every epilogue thread has read the P tile
+        if (tid == 0) bar_arrive(&empty[s]);
+      } else {
+        bar_wait(acc_full, ni & 1u);
+        ++ni;
+        fence_after();
+#pragma unroll
+        for (int q = 0; q < 2; ++q) {
+          float a0[16], a1[16], a2[16], a3[16], cc[16];
+          tmem_ld16(tl + 0 * TS + q * 16, a0);
+          tmem_ld16(tl + 1 * TS + q * 16, a1);
+          tmem_ld16(tl + 2 * TS + q * 16, a2);
+          tmem_ld16(tl + 3 * TS + q * 16, a3);
+          tmem_ld16(tl + 4 * TS + q * 16, cc);
+          tmem_wait_ld();
+#pragma unroll
+          for (int i = 0; i < 16; ++i) dv[q * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
+        }
+        fence_before();
+        __syncwarp();
+        if (lane == 0) bar_arrive(acc_empty);  // the MMAs of the next internal phase may overwrite them
       }
-      fence_before();
-      __syncwarp();
-      if (lane == 0) bar_arrive(acc_empty);  // the MMAs of phase g+1 may overwrite them
       if (b == 0) {
 #pragma unroll
         for (int k = 0; k < 8; ++k)
