@@ -42,6 +42,64 @@ __global__ void k_transition(int s, int s_pad, int C, const double *__restrict__
   }
 }
 
+// K1 for the codon state space (s_pad = 64): one block per listed matrix, all
+// categories.  The same sum as above, register-tiled: thread (ty, tx) of a
+// 16 x 16 block owns the 4 x 4 outputs z in [4ty, 4ty+4), x in [4tx, 4tx+4),
+// and per k reads 4 consecutive V^T[k][z] and 4 consecutive Vinv[k][x]
+// (two 16-byte shared loads each) for 16 fp64 FMAs -- 4 loads per 16 FMAs
+// instead of 2 per FMA.  V, Vinv are zero-padded to 64 x 64 in shared memory,
+// so padding outputs come out exactly zero.
+template <typename T>
+__global__ void __launch_bounds__(256)
+k_transition64(int s, int C, const double *__restrict__ eig, const double *__restrict__ rates,
+               const int32_t *__restrict__ idx, const double *__restrict__ tlen, T *__restrict__ P) {
+  extern __shared__ double sm[];
+  double *Vt = sm;              // [64 k][64 z]
+  double *Vi = sm + 64 * 64;    // [64 k][64 x]
+  double *ex = sm + 2 * 64 * 64;  // [C][64]
+  const int m = blockIdx.x, tid = threadIdx.x;
+  const double *lam = eig + 2 * s * s;
+  for (int i = tid; i < 64 * 64; i += 256) {
+    const int a = i >> 6, b = i & 63;  // a = row, b = column of the padded matrix
+    Vt[b * 64 + a] = (a < s && b < s) ? eig[a * s + b] : 0.0;        // V[a][b] -> Vt[k=b][z=a]
+    Vi[i] = (a < s && b < s) ? eig[s * s + a * s + b] : 0.0;         // Vinv[k=a][x=b]
+  }
+  const double t = tlen[m];
+  for (int i = tid; i < C * 64; i += 256) {
+    const int c = i >> 6, k = i & 63;
+    ex[i] = k < s ? exp(lam[k] * rates[c] * t) : 0.0;
+  }
+  __syncthreads();
+  const int z0 = (tid >> 4) * 4, x0 = (tid & 15) * 4;
+  for (int c = 0; c < C; ++c) {
+    double acc[4][4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc[i][j] = 0.0;
+    const double *e = ex + c * 64;
+#pragma unroll 4
+    for (int k = 0; k < s; ++k) {
+      const double2 va = *reinterpret_cast<const double2 *>(Vt + k * 64 + z0);
+      const double2 vb = *reinterpret_cast<const double2 *>(Vt + k * 64 + z0 + 2);
+      const double2 wa = *reinterpret_cast<const double2 *>(Vi + k * 64 + x0);
+      const double2 wb = *reinterpret_cast<const double2 *>(Vi + k * 64 + x0 + 2);
+      const double ek = e[k];
+      const double a[4] = {va.x * ek, va.y * ek, vb.x * ek, vb.y * ek};
+      const double b[4] = {wa.x, wa.y, wb.x, wb.y};
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
+    }
+    T *out = P + ((size_t)idx[m] * C + c) * 64 * 64;
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) out[(z0 + i) * 64 + x0 + j] = (T)acc[i][j];
+  }
+}
+
 // ---------------------------------------------------------------------- K5
 __global__ void k_accumulate(const int32_t *__restrict__ scale, int p_pad,
                              const int32_t *__restrict__ idx, int count, int32_t *__restrict__ cum,
@@ -176,6 +234,22 @@ int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *
                                int count, void *d_P, void *stream) {
   if (count <= 0) return 0;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (s_pad == 64) {  // codon: register-tiled, one block per matrix
+    const size_t smem64 = sizeof(double) * (2 * 64 * 64 + (size_t)c * 64);
+    for (int o = 0; o < count; o += 0x7fffffff) {
+      const int n = count - o;
+      if (prec == 32) {
+        cudaFuncSetAttribute(k_transition64<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
+        k_transition64<float><<<n, 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx + o, d_t + o,
+                                                       static_cast<float *>(d_P));
+      } else {
+        cudaFuncSetAttribute(k_transition64<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
+        k_transition64<double><<<n, 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx + o, d_t + o,
+                                                        static_cast<double *>(d_P));
+      }
+    }
+    return (int)cudaGetLastError();
+  }
   const size_t smem = sizeof(double) * (2 * s * s + s);
   const int threads = (s <= 4) ? 32 : 256;
   for (int o = 0; o < count; o += 65535) {
