@@ -51,6 +51,7 @@ struct Instance {
   std::vector<char> has_states;
   uint8_t *d_states = nullptr;           // [n_tips][p_pad]
   char *d_P = nullptr;                   // [n_mat][c][s_pad][s_pad]
+  float *d_Plo = nullptr;                // fp32 codon: tf32 low parts of d_P (3xTF32 operand), same layout
   int32_t *d_scale = nullptr;            // [n_scale][p_pad]
   double *d_eig = nullptr;               // [n_eig][2 s^2 + s]
   double *d_rates = nullptr;             // [n_eig][c] (per model / partition)
@@ -91,7 +92,7 @@ struct Instance {
   rrl_profile prof{};
 
   // TMA descriptors of the internal-partials and matrix slabs (61-state fp32, K3-TC5)
-  CUtensorMap tmap_partials{}, tmap_P{};
+  CUtensorMap tmap_partials{}, tmap_P{}, tmap_Plo{};
   bool tmaps_ok = false;
 };
 
@@ -196,7 +197,7 @@ void destroy(Instance *I) {
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
                   I->d_catw,     I->d_freqs,  I->d_pw,   I->d_site,  I->d_block, I->d_out, I->d_count,
-                  I->d_midx,     I->d_t,      I->d_sidx, I->d_ops};
+                  I->d_midx,     I->d_t,      I->d_sidx, I->d_ops,  I->d_Plo};
   for (void *q : ptrs)
     if (q) cudaFree(q);
   if (I->h_ops) cudaFreeHost(I->h_ops);
@@ -371,7 +372,13 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
       const CUresult r2 = enc(&I->tmap_P, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, I->d_P, gP, sP, bP, es,
                               CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-      I->tmaps_ok = (r1 == CUDA_SUCCESS && r2 == CUDA_SUCCESS);
+      const size_t pbytes = (size_t)matrix_count * I->mat_elems * I->elt;
+      CKC(cudaMalloc(&I->d_Plo, pbytes));
+      CKC(cudaMemset(I->d_Plo, 0, pbytes));
+      const CUresult r3 = enc(&I->tmap_Plo, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, I->d_Plo, gP, sP, bP, es,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+      I->tmaps_ok = (r1 == CUDA_SUCCESS && r2 == CUDA_SUCCESS && r3 == CUDA_SUCCESS);
     }
   }
   CKC(cudaMallocHost(&I->h_out, sizeof(double)));
@@ -585,7 +592,7 @@ int rrl_update_transition_matrices(int inst, int eigen_idx, const int32_t *matri
     Timed tm(I, 1);
     CKL(launch_transition_matrices(I->prec, I->s, I->s_pad, I->c, I->d_eig + eig_sz * eigen_idx,
                                    I->d_rates + (size_t)eigen_idx * I->c, I->d_midx, I->d_t, count, I->d_P,
-                                   I->stream));
+                                   I->d_Plo, I->stream));
   }
   I->prof.matrices_launches += (count + 65534) / 65535;
   I->prof.kernel_launches += (count + 65534) / 65535;
@@ -607,6 +614,9 @@ int rrl_set_transition_matrix(int inst, int idx, const double *P) {
       }
   CK(cudaMemcpyAsync(I->d_P + (size_t)idx * h.size(), h.data(), h.size(), cudaMemcpyHostToDevice,
                      I->stream));
+  if (I->d_Plo)  // keep the 3xTF32 low parts of this matrix in step (device split, like K1's)
+    CKL(launch_split_tf32(reinterpret_cast<const float *>(I->d_P + (size_t)idx * h.size()),
+                         I->d_Plo + (size_t)idx * I->mat_elems, I->mat_elems, I->stream));
   CK(cudaStreamSynchronize(I->stream));
   return RRL_SUCCESS;
 }
@@ -799,7 +809,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
         e = (int)cudaErrorNotSupported;
         if (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT) && I->tmaps_ok)  // TMA-fed tcgen05 (c <= 4)
           e = launch_update_partials_codon_tc5(I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax, I->p_pad,
-                                               &I->tmap_partials, &I->tmap_P, I->stream);
+                                               &I->tmap_partials, &I->tmap_P, &I->tmap_Plo, I->stream);
         if (e == (int)cudaErrorNotSupported && I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))
           e = launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, pmax, I->p_pad, I->stream);
         if (e == (int)cudaErrorNotSupported)

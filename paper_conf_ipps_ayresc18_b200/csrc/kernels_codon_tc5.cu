@@ -14,8 +14,9 @@
 //    stages, 128-byte swizzled -- the canonical SWIZZLE_128B K-major UMMA
 //    layout, so the raw fp32 tile IS the tf32 "hi" operand (the tensor core
 //    reads the top 19 bits of each 32-bit element);
-//  * converters (warps 8-11): the tf32 "lo" parts, lo = rn_tf32(x - hi(x)),
-//    elementwise in place of layout (same swizzled offsets), for A and P;
+//  * converters (warps 8-11): the tf32 "lo" parts of the child tile,
+//    lo = rn_tf32(x - hi(x)), elementwise in place of layout (same swizzled
+//    offsets); P's lo parts come precomputed from K1 (a second slab, TMA'd);
 //  * a tip child (uint8 states) is no contraction at all: sum_x P[z][x] [x = obs]
 //    = P[z][obs], so its phase lands only the raw P tile and the epilogue
 //    gathers the column from shared memory (row sums for a missing state) --
@@ -142,7 +143,8 @@ __device__ inline int frexp_e(float m) {
 template <int C>
 __global__ void __launch_bounds__(kThr, 1)
 k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p_pad,
-                     const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmP) {
+                     const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmP,
+                     const __grid_constant__ CUtensorMap tmPlo) {
   static_assert(kProdCol + (C - 1) * TS <= kTmemCols, "parked products must fit TMEM");
   extern __shared__ __align__(1024) unsigned char sm[];
   uint64_t *tma_full = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);  // [2]
@@ -173,6 +175,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tmA) : "memory");
     asm volatile("prefetch.tensormap [%0];" ::"l"(&tmP) : "memory");
+    asm volatile("prefetch.tensormap [%0];" ::"l"(&tmPlo) : "memory");
   }
   fence_before();
   __syncthreads();
@@ -196,10 +199,12 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         const int buf = b == 0 ? op.buf1 : op.buf2, mat = b == 0 ? op.mat1 : op.mat2;
         bar_wait(&empty[s], ((uint32_t)(g >> 1) & 1u) ^ 1u);  // MMAs of phase g-2 are done
         const uint32_t st = sbase + s * ST_BYTES;
-        bar_expect(&tma_full[s], (tip ? 0u : 32768u) + 16384u);
-        if (!tip) {
+        bar_expect(&tma_full[s], (tip ? 0u : 32768u + 16384u) + 16384u);
+        if (!tip) {  // child tile + the matrix's precomputed tf32 low parts (written by K1)
           tma4(st + ST_AHI, &tmA, 0, op.pat0 + p0, c, buf, &tma_full[s]);
           tma4(st + ST_AHI + 16384, &tmA, 32, op.pat0 + p0, c, buf, &tma_full[s]);
+          tma4(st + ST_BLO, &tmPlo, 0, 0, c, mat, &tma_full[s]);
+          tma4(st + ST_BLO + 8192, &tmPlo, 32, 0, c, mat, &tma_full[s]);
         }
         tma4(st + ST_BHI, &tmP, 0, 0, c, mat, &tma_full[s]);
         tma4(st + ST_BHI + 8192, &tmP, 32, 0, c, mat, &tma_full[s]);
@@ -245,17 +250,15 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       unsigned char *st = sm + s * ST_BYTES;
       bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
       if (!tip) {  // a tip phase only lands P for the epilogue's gather: nothing to convert
-#pragma unroll 4
-        for (int i = ct; i < TM * 16; i += kConvThr) {  // lo of every 16-byte chunk, same swizzled offset
-          const float4 v = *reinterpret_cast<const float4 *>(st + ST_AHI + i * 16);
-          *reinterpret_cast<float4 *>(st + ST_ALO + i * 16) =
-              make_float4(lo_tf32(v.x), lo_tf32(v.y), lo_tf32(v.z), lo_tf32(v.w));
-        }
-#pragma unroll 2
-        for (int i = ct; i < TS * 16; i += kConvThr) {
-          const float4 v = *reinterpret_cast<const float4 *>(st + ST_BHI + i * 16);
-          *reinterpret_cast<float4 *>(st + ST_BLO + i * 16) =
-              make_float4(lo_tf32(v.x), lo_tf32(v.y), lo_tf32(v.z), lo_tf32(v.w));
+#pragma unroll
+        for (int u = 0; u < TM * 16 / kConvThr; u += 8) {  // lo of every 16-byte chunk, same swizzled offset
+          float4 v[8];
+#pragma unroll
+          for (int q = 0; q < 8; ++q) v[q] = *reinterpret_cast<const float4 *>(st + ST_AHI + (ct + (u + q) * kConvThr) * 16);
+#pragma unroll
+          for (int q = 0; q < 8; ++q)
+            *reinterpret_cast<float4 *>(st + ST_ALO + (ct + (u + q) * kConvThr) * 16) =
+                make_float4(lo_tf32(v[q].x), lo_tf32(v[q].y), lo_tf32(v[q].z), lo_tf32(v[q].w));
         }
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
@@ -409,7 +412,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
 
 template <int C>
 int launch_tc5(const DevOp *d_ops, int nops, int p, int p_pad, const CUtensorMap *tA, const CUtensorMap *tP,
-               cudaStream_t st) {
+               const CUtensorMap *tPlo, cudaStream_t st) {
   static int nsm = 0;
   if (nsm == 0) {
     cudaError_t e = cudaFuncSetAttribute(k_partials_codon_tc5<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -433,13 +436,15 @@ int launch_tc5(const DevOp *d_ops, int nops, int p, int p_pad, const CUtensorMap
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  return (int)cudaLaunchKernelEx(&cfg, k_partials_codon_tc5<C>, d_ops, ntiles, (int)total, p_pad, *tA, *tP);
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_codon_tc5<C>, d_ops, ntiles, (int)total, p_pad, *tA, *tP,
+                                 *tPlo);
 }
 
 }  // namespace
 
 int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
-                                     int p_pad, const void *tmap_partials, const void *tmap_P, void *stream) {
+                                     int p_pad, const void *tmap_partials, const void *tmap_P,
+                                     const void *tmap_Plo, void *stream) {
   // every child must live in the tensor-mapped slab (internal buffers) or be tip states
   for (int i = 0; i < nops; ++i)
     if ((!(h_ops[i].flags & OP_TIP1) && h_ops[i].buf1 < 0) || (!(h_ops[i].flags & OP_TIP2) && h_ops[i].buf2 < 0))
@@ -447,10 +452,11 @@ int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_o
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const CUtensorMap *tA = static_cast<const CUtensorMap *>(tmap_partials);
   const CUtensorMap *tP = static_cast<const CUtensorMap *>(tmap_P);
+  const CUtensorMap *tPlo = static_cast<const CUtensorMap *>(tmap_Plo);
   switch (c) {
-    case 1: return launch_tc5<1>(d_ops, nops, p, p_pad, tA, tP, st);
-    case 2: return launch_tc5<2>(d_ops, nops, p, p_pad, tA, tP, st);
-    case 4: return launch_tc5<4>(d_ops, nops, p, p_pad, tA, tP, st);
+    case 1: return launch_tc5<1>(d_ops, nops, p, p_pad, tA, tP, tPlo, st);
+    case 2: return launch_tc5<2>(d_ops, nops, p, p_pad, tA, tP, tPlo, st);
+    case 4: return launch_tc5<4>(d_ops, nops, p, p_pad, tA, tP, tPlo, st);
     default: return (int)cudaErrorNotSupported;
   }
 }

@@ -42,42 +42,47 @@ __global__ void k_transition(int s, int s_pad, int C, const double *__restrict__
   }
 }
 
-// K1 for the codon state space (s_pad = 64): one block per listed matrix, all
-// categories.  The same sum as above, register-tiled: thread (ty, tx) of a
+// K1 for the codon state space (s_pad = 64): one block per (listed matrix,
+// category).  The same sum as above, register-tiled: thread (ty, tx) of a
 // 16 x 16 block owns the 4 x 4 outputs z in [4ty, 4ty+4), x in [4tx, 4tx+4),
 // and per k reads 4 consecutive V^T[k][z] and 4 consecutive Vinv[k][x]
 // (two 16-byte shared loads each) for 16 fp64 FMAs -- 4 loads per 16 FMAs
 // instead of 2 per FMA.  V, Vinv are zero-padded to 64 x 64 in shared memory,
-// so padding outputs come out exactly zero.
+// so padding outputs come out exactly zero.  With Plo (fp32 codon instances
+// feeding the tcgen05 kernel) the tf32 low part of every stored entry is
+// written beside it, once per matrix instead of once per pattern tile.
+__device__ inline float tf32_lo(float x) {  // rn_tf32(x - trunc_tf32(x)), the 3xTF32 low part
+  const float hi = __uint_as_float(__float_as_uint(x) & 0xffffe000u);
+  return __uint_as_float((__float_as_uint(x - hi) + 0x1000u) & 0xffffe000u);
+}
+
 template <typename T>
 __global__ void __launch_bounds__(256)
 k_transition64(int s, int C, const double *__restrict__ eig, const double *__restrict__ rates,
-               const int32_t *__restrict__ idx, const double *__restrict__ tlen, T *__restrict__ P) {
+               const int32_t *__restrict__ idx, const double *__restrict__ tlen, T *__restrict__ P,
+               float *__restrict__ Plo) {
   extern __shared__ double sm[];
   double *Vt = sm;              // [64 k][64 z]
   double *Vi = sm + 64 * 64;    // [64 k][64 x]
   double *ex = sm + 2 * 64 * 64;  // [C][64]
-  const int m = blockIdx.x, tid = threadIdx.x;
+  const int m = blockIdx.x, c = blockIdx.y, tid = threadIdx.x;
   const double *lam = eig + 2 * s * s;
   for (int i = tid; i < 64 * 64; i += 256) {
     const int a = i >> 6, b = i & 63;  // a = row, b = column of the padded matrix
     Vt[b * 64 + a] = (a < s && b < s) ? eig[a * s + b] : 0.0;        // V[a][b] -> Vt[k=b][z=a]
     Vi[i] = (a < s && b < s) ? eig[s * s + a * s + b] : 0.0;         // Vinv[k=a][x=b]
   }
-  const double t = tlen[m];
-  for (int i = tid; i < C * 64; i += 256) {
-    const int c = i >> 6, k = i & 63;
-    ex[i] = k < s ? exp(lam[k] * rates[c] * t) : 0.0;
-  }
+  const double rt = rates[c] * tlen[m];
+  for (int k = tid; k < 64; k += 256) ex[k] = k < s ? exp(lam[k] * rt) : 0.0;
   __syncthreads();
   const int z0 = (tid >> 4) * 4, x0 = (tid & 15) * 4;
-  for (int c = 0; c < C; ++c) {
+  {
     double acc[4][4];
 #pragma unroll
     for (int i = 0; i < 4; ++i)
 #pragma unroll
       for (int j = 0; j < 4; ++j) acc[i][j] = 0.0;
-    const double *e = ex + c * 64;
+    const double *e = ex;
 #pragma unroll 4
     for (int k = 0; k < s; ++k) {
       const double2 va = *reinterpret_cast<const double2 *>(Vt + k * 64 + z0);
@@ -92,12 +97,21 @@ k_transition64(int s, int C, const double *__restrict__ eig, const double *__res
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[i][j] = fma(a[i], b[j], acc[i][j]);
     }
-    T *out = P + ((size_t)idx[m] * C + c) * 64 * 64;
+    const size_t off = ((size_t)idx[m] * C + c) * 64 * 64;
 #pragma unroll
     for (int i = 0; i < 4; ++i)
 #pragma unroll
-      for (int j = 0; j < 4; ++j) out[(z0 + i) * 64 + x0 + j] = (T)acc[i][j];
+      for (int j = 0; j < 4; ++j) {
+        const T v = (T)acc[i][j];
+        P[off + (z0 + i) * 64 + x0 + j] = v;
+        if (Plo != nullptr) Plo[off + (z0 + i) * 64 + x0 + j] = tf32_lo((float)v);
+      }
   }
+}
+
+__global__ void k_split_tf32(const float *__restrict__ x, float *__restrict__ lo, size_t n) {
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n; i += (size_t)gridDim.x * blockDim.x)
+    lo[i] = tf32_lo(x[i]);
 }
 
 // ---------------------------------------------------------------------- K5
@@ -231,22 +245,20 @@ k_edge(const T *__restrict__ Lp, const void *__restrict__ child, int child_is_ti
 
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
-                               int count, void *d_P, void *stream) {
+                               int count, void *d_P, void *d_Plo, void *stream) {
   if (count <= 0) return 0;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (s_pad == 64) {  // codon: register-tiled, one block per matrix
-    const size_t smem64 = sizeof(double) * (2 * 64 * 64 + (size_t)c * 64);
-    for (int o = 0; o < count; o += 0x7fffffff) {
-      const int n = count - o;
-      if (prec == 32) {
-        cudaFuncSetAttribute(k_transition64<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
-        k_transition64<float><<<n, 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx + o, d_t + o,
-                                                       static_cast<float *>(d_P));
-      } else {
-        cudaFuncSetAttribute(k_transition64<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
-        k_transition64<double><<<n, 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx + o, d_t + o,
-                                                        static_cast<double *>(d_P));
-      }
+    const size_t smem64 = sizeof(double) * (2 * 64 * 64 + 64);
+    if (prec == 32) {
+      cudaFuncSetAttribute(k_transition64<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
+      k_transition64<float><<<dim3(count, c), 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx, d_t,
+                                                                 static_cast<float *>(d_P),
+                                                                 static_cast<float *>(d_Plo));
+    } else {
+      cudaFuncSetAttribute(k_transition64<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
+      k_transition64<double><<<dim3(count, c), 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx, d_t,
+                                                                  static_cast<double *>(d_P), nullptr);
     }
     return (int)cudaGetLastError();
   }
@@ -306,6 +318,13 @@ int launch_edge_lnl(int prec, int s, int s_pad, int c, const void *par, const vo
     k_edge<double><<<nblocks, 256, 0, st>>>(static_cast<const double *>(par), child, child_is_tip,
                                             static_cast<const double *>(P), s, s_pad, c, d_w, d_pi,
                                             cum_p, cum_c, d_pw, p, p_pad, d_site, d_block, d_count, d_out);
+  return (int)cudaGetLastError();
+}
+
+int launch_split_tf32(const float *x, float *lo, size_t n, void *stream) {
+  if (n == 0) return 0;
+  const size_t blocks = (n + 255) / 256;
+  k_split_tf32<<<(unsigned)(blocks < 4096 ? blocks : 4096), 256, 0, static_cast<cudaStream_t>(stream)>>>(x, lo, n);
   return (int)cudaGetLastError();
 }
 

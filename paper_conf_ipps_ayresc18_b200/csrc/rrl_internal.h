@@ -51,11 +51,14 @@ int launch_update_partials_codon_tc(int c, const DevOp *d_ops, int nops, int p, 
 // partials slab / matrix slab tensor maps (opaque 128-byte CUtensorMap values
 // passed as void*), converter warps derive the tf32 lo parts in shared memory.
 // cudaErrorNotSupported when a child of the set is not in the slab.
+// tf32 low parts lo = rn(x - trunc_tf32(x)) of n fp32 values (the 3xTF32 split of P).
+int launch_split_tf32(const float *x, float *lo, size_t n, void *stream);
 int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
-                                     int p_pad, const void *tmap_partials, const void *tmap_P, void *stream);
+                                     int p_pad, const void *tmap_partials, const void *tmap_P,
+                                     const void *tmap_Plo, void *stream);
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
-                               int count, void *d_P, void *stream);
+                               int count, void *d_P, void *d_Plo, void *stream);
 int launch_accumulate_scale(const int32_t *d_scale, int p_pad, const int32_t *d_idx, int count,
                             int32_t *d_cum, int p, void *stream);
 int launch_root_lnl(int prec, int s, int s_pad, int c, const void *root, const double *d_w,
