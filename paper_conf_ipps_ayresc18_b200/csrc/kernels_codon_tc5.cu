@@ -21,15 +21,16 @@
 //    = P[z][obs], so its phase lands only the raw P tile and the epilogue
 //    gathers the column from shared memory (row sums for a missing state) --
 //    no conversion, no MMA, no TMEM traffic;
-//  * MMA issuer (warp 13, one lane): per K-step of 8, hi*hi into one of four
-//    main accumulators and hi*lo + lo*hi into a correction accumulator (the
-//    accumulation-precision scheme measured in DESIGN.md), tcgen05.commit to
-//    the stage's `empty` and to `acc_full`;
+//  * MMA issuer (warp 13, one lane): per K-step of 8, one N = 128 MMA
+//    A_hi.[P_hi|P_lo]^T into [main_h | corr_h] and one N = 64 MMA A_lo.P_hi^T
+//    into corr_h (h = K-half: two main accumulators, never mixed with the
+//    corrections -- the accumulation-precision reading in DESIGN.md),
+//    tcgen05.commit to the stage's `empty` and to `acc_full`;
 //  * epilogue (warps 0-7: TMEM lane quarter w%4, column half w/4): sums the
-//    five accumulators (tcgen05.ld 32x32b.x16), releases `acc_empty`, parks
-//    child 1 in shared memory, forms the product with child 2, parks it in
-//    TMEM until the tile's last category, then scales by 2^-e and writes every
-//    category once, coalesced, through a swizzled staging tile.
+//    four accumulators (tcgen05.ld 32x32b.x16), releases `acc_empty`, parks
+//    child 1 in the category's TMEM slot, forms the product with child 2, parks
+//    it in the same slot until the tile's last category, then scales by 2^-e
+//    and writes every category once, coalesced, through a swizzled staging tile.
 // Compared with K3-TC (kernels_codon_tc.cu) the SM no longer moves the child
 // tile through registers: per phase it only writes the lo halves.
 #include <cuda.h>
@@ -49,29 +50,32 @@ constexpr int kEpiThr = 256;                 // warps 0-7
 constexpr int kConvThr = 128;                // warps 8-11
 constexpr int kProdWarp = 12, kMmaWarp = 13;
 constexpr int kThr = 14 * 32;
-// one stage: A hi (2 x 16 KB halves k 0-31 / 32-63), A lo, P hi (2 x 8 KB), P lo
-constexpr int ST_AHI = 0, ST_ALO = 32768, ST_BHI = 65536, ST_BLO = 81920, ST_BYTES = 98304;
+// one stage: A hi (2 x 16 KB halves k 0-31 / 32-63), A lo, then B = per K-half h
+// [P hi rows 0-63 | P lo rows 0-63] (16 KB), so one N = 128 MMA reads A hi once
+// for both hi.hi and hi.lo.
+constexpr int ST_AHI = 0, ST_ALO = 32768, ST_B = 65536, ST_BYTES = 98304;
 constexpr int SMEM_S1 = 2 * ST_BYTES;                  // epilogue staging tile (32 KB)
 constexpr int SMEM_MX = SMEM_S1 + TM * TS * 4;         // row maxima / scale [2][128]
 constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 8 mbarriers
 constexpr int SMEM_TMEM = SMEM_BAR + 8 * 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 16;
-constexpr int kTmemCols = 512;    // 4 main + 1 correction accumulator (5 x 64) ...
-constexpr int kProdCol = 5 * TS;  // ... + parked products of categories 0..C-2
+constexpr int kTmemCols = 512;    // per K-half h: [main_h | corr_h] (4 x 64) ...
+constexpr int kProdCol = 4 * TS;  // ... + one 64-column slot per category (child 1, then the product)
 
 __device__ inline uint32_t sa(const void *p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
 __device__ inline uint64_t desc_sw128(uint32_t saddr) {  // K-major, 128-byte swizzle, 8-row atoms of 1 KB
   return (uint64_t)((saddr & 0x3FFFFu) >> 4) | ((uint64_t)1 << 16) | ((uint64_t)(1024 >> 4) << 32) |
          ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
 }
-constexpr uint32_t kIdesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(TS >> 3) << 17) |
-                            ((uint32_t)(TM >> 4) << 24);  // kind::tf32, D f32, K-major A/B, N 64, M 128
+__host__ __device__ constexpr uint32_t idesc_tf32(int n) {  // kind::tf32, D f32, K-major A/B, M 128, N n
+  return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(n >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
+}
 
-__device__ inline void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t acc) {
+__device__ inline void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t acc) {
   asm volatile(
       "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
       "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
-      "l"(a), "l"(b), "r"(kIdesc), "r"(acc));
+      "l"(a), "l"(b), "r"(idesc), "r"(acc));
 }
 __device__ inline void commit(uint64_t *bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(sa(bar))
@@ -145,7 +149,7 @@ __global__ void __launch_bounds__(kThr, 1)
 k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p_pad,
                      const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmP,
                      const __grid_constant__ CUtensorMap tmPlo) {
-  static_assert(kProdCol + (C - 1) * TS <= kTmemCols, "parked products must fit TMEM");
+  static_assert(kProdCol + C * TS <= kTmemCols, "category slots must fit TMEM");
   extern __shared__ __align__(1024) unsigned char sm[];
   uint64_t *tma_full = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);  // [2]
   uint64_t *conv_full = tma_full + 2;                                 // [2]
@@ -203,11 +207,11 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         if (!tip) {  // child tile + the matrix's precomputed tf32 low parts (written by K1)
           tma4(st + ST_AHI, &tmA, 0, op.pat0 + p0, c, buf, &tma_full[s]);
           tma4(st + ST_AHI + 16384, &tmA, 32, op.pat0 + p0, c, buf, &tma_full[s]);
-          tma4(st + ST_BLO, &tmPlo, 0, 0, c, mat, &tma_full[s]);
-          tma4(st + ST_BLO + 8192, &tmPlo, 32, 0, c, mat, &tma_full[s]);
+          tma4(st + ST_B + 8192, &tmPlo, 0, 0, c, mat, &tma_full[s]);
+          tma4(st + ST_B + 16384 + 8192, &tmPlo, 32, 0, c, mat, &tma_full[s]);
         }
-        tma4(st + ST_BHI, &tmP, 0, 0, c, mat, &tma_full[s]);
-        tma4(st + ST_BHI + 8192, &tmP, 32, 0, c, mat, &tma_full[s]);
+        tma4(st + ST_B, &tmP, 0, 0, c, mat, &tma_full[s]);
+        tma4(st + ST_B + 16384, &tmP, 32, 0, c, mat, &tma_full[s]);
       }
     }
   } else if (warp == kMmaWarp) {
@@ -224,17 +228,18 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         ++ni;
         fence_after();
         const uint32_t st = sbase + s * ST_BYTES;
+        // per K-step of 8: A_hi . [P_hi | P_lo]^T (N = 128) -> [main_h | corr_h], then
+        // A_lo . P_hi^T (N = 64) -> corr_h; main and the ~2^-11-smaller corrections
+        // never share an accumulator (tf32 accumulation reading).
 #pragma unroll
         for (int kk = 0; kk < TS / 8; ++kk) {
           const int h = kk >> 2, kin = kk & 3;
           const uint64_t ah = desc_sw128(st + ST_AHI + h * 16384 + kin * 32);
           const uint64_t al = desc_sw128(st + ST_ALO + h * 16384 + kin * 32);
-          const uint64_t bh = desc_sw128(st + ST_BHI + h * 8192 + kin * 32);
-          const uint64_t bl = desc_sw128(st + ST_BLO + h * 8192 + kin * 32);
-          const uint32_t dmain = tmem + (uint32_t)((kk >> 1) * TS), dcorr = tmem + (uint32_t)(4 * TS);
-          mma_tf32(dmain, ah, bh, (kk & 1) ? 1u : 0u);
-          mma_tf32(dcorr, ah, bl, kk > 0 ? 1u : 0u);
-          mma_tf32(dcorr, al, bh, 1u);
+          const uint64_t bb = desc_sw128(st + ST_B + h * 16384 + kin * 32);
+          const uint32_t d = tmem + (uint32_t)(h * 2 * TS);
+          mma_tf32(d, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);
+          mma_tf32(d + TS, al, bb, idesc_tf32(TS), 1u);
         }
         commit(&empty[s]);  // stage free once these MMAs completed
         commit(acc_full);   // accumulators ready for the epilogue
@@ -273,7 +278,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     auto s1 = [&](int row, int k) -> float4 * {  // 16 x 16-byte chunks per row, chunk k at k ^ (row & 15)
       return reinterpret_cast<float4 *>(S1 + row * TS + 4 * (k ^ (row & 15)));
     };
-    float m = 0.f;  // child 1 of the current category waits in this thread's own S1 half-row
+    float m = 0.f;  // running max over (c, z) of this thread's row half
     uint32_t ni = 0;  // internal-child phases consumed (accumulator barrier parity)
     for (int g = 0; g < nphase; ++g) {
       const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
@@ -289,11 +294,11 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         // position chunk ^ (z&7) of half x>>5). A missing state (code >= 61) is the row sum.
         const int s = g & 1;
         bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
-        const unsigned char *pt = sm + s * ST_BYTES + ST_BHI;
+        const unsigned char *pt = sm + s * ST_BYTES + ST_B;  // P hi of K-half h at h * 16 KB
         const uint8_t *states = static_cast<const uint8_t *>(b == 0 ? op.in1 : op.in2);  // range-offset
         const unsigned sv = valid ? (unsigned)states[pp] : 0u;
         if (sv < (unsigned)kS61) {
-          const unsigned char *base = pt + (sv >> 5) * 8192 + (sv & 3) * 4;
+          const unsigned char *base = pt + (sv >> 5) * 16384 + (sv & 3) * 4;
           const unsigned j = (sv & 31) >> 2;
 #pragma unroll
           for (int i = 0; i < 32; ++i) {
@@ -305,7 +310,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
           for (int i = 0; i < 32; ++i) dv[i] = 0.f;
 #pragma unroll 1
           for (int x = 0; x < kS61; ++x) {
-            const unsigned char *base = pt + (x >> 5) * 8192 + (x & 3) * 4;
+            const unsigned char *base = pt + (x >> 5) * 16384 + (x & 3) * 4;
             const unsigned j = (unsigned)(x & 31) >> 2;
 #pragma unroll
             for (int i = 0; i < 32; ++i) {
@@ -322,35 +327,42 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         fence_after();
 #pragma unroll
         for (int q = 0; q < 2; ++q) {
-          float a0[16], a1[16], a2[16], a3[16], cc[16];
-          tmem_ld16(tl + 0 * TS + q * 16, a0);
-          tmem_ld16(tl + 1 * TS + q * 16, a1);
-          tmem_ld16(tl + 2 * TS + q * 16, a2);
-          tmem_ld16(tl + 3 * TS + q * 16, a3);
-          tmem_ld16(tl + 4 * TS + q * 16, cc);
+          float m0[16], c0[16], m1[16], c1[16];
+          tmem_ld16(tl + 0 * TS + q * 16, m0);
+          tmem_ld16(tl + 1 * TS + q * 16, c0);
+          tmem_ld16(tl + 2 * TS + q * 16, m1);
+          tmem_ld16(tl + 3 * TS + q * 16, c1);
           tmem_wait_ld();
 #pragma unroll
-          for (int i = 0; i < 16; ++i) dv[q * 16 + i] = ((a0[i] + a1[i]) + (a2[i] + a3[i])) + cc[i];
+          for (int i = 0; i < 16; ++i) dv[q * 16 + i] = (m0[i] + m1[i]) + (c0[i] + c1[i]);
         }
         fence_before();
         __syncwarp();
         if (lane == 0) bar_arrive(acc_empty);  // the MMAs of the next internal phase may overwrite them
       }
-      if (b == 0) {
-#pragma unroll
-        for (int k = 0; k < 8; ++k)
-          *s1(r, h * 8 + k) = make_float4(dv[4 * k], dv[4 * k + 1], dv[4 * k + 2], dv[4 * k + 3]);
+      const uint32_t slot = tl + (uint32_t)(kProdCol + c * TS);  // this category's TMEM slot
+      if (b == 0) {  // child 1 waits in the slot until child 2's phase
+        tmem_st16(slot, dv);
+        tmem_st16(slot + 16, dv + 16);
+        tmem_wait_st();
         continue;
       }
+      {
+        float w0[16], w1[16];
+        tmem_ld16(slot, w0);
+        tmem_ld16(slot + 16, w1);
+        tmem_wait_ld();
 #pragma unroll
-      for (int k = 0; k < 8; ++k) {
-        const float4 w = *s1(r, h * 8 + k);
-        dv[4 * k] *= w.x; dv[4 * k + 1] *= w.y; dv[4 * k + 2] *= w.z; dv[4 * k + 3] *= w.w;
-        m = fmaxf(m, fmaxf(fmaxf(dv[4 * k], dv[4 * k + 1]), fmaxf(dv[4 * k + 2], dv[4 * k + 3])));
+        for (int i = 0; i < 16; ++i) {
+          dv[i] *= w0[i];
+          dv[16 + i] *= w1[i];
+        }
+#pragma unroll
+        for (int i = 0; i < 32; ++i) m = fmaxf(m, dv[i]);
       }
-      if (c < C - 1) {  // park the unscaled product until the tile's exponent is known
-        tmem_st16(tl + (uint32_t)(kProdCol + c * TS), dv);
-        tmem_st16(tl + (uint32_t)(kProdCol + c * TS + 16), dv + 16);
+      if (c < C - 1) {  // park the unscaled product (in place of child 1) until the tile's exponent is known
+        tmem_st16(slot, dv);
+        tmem_st16(slot + 16, dv + 16);
         tmem_wait_st();
         continue;
       }
@@ -401,8 +413,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
             *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
         }
       }
-      named_sync(1, kEpiThr);  // staging reads done before rows are reused for child 1
-      m = 0.f;
+      m = 0.f;  // (the next tile's first staging write waits at the loop's first barrier)
     }
   }
   fence_before();
