@@ -17,13 +17,17 @@ HERE = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(HERE)
 CSRC = os.path.join(HERE, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
-BUILD = os.path.join(ROOT, "build", "rrl")
+# Dev variants (e.g. tools/trace_tc5.py): RRL_NVCC_EXTRA adds nvcc flags and
+# RRL_BUILD_TAG builds into build/rrl-<tag> and _lib/librrl-<tag>.so instead.
+_TAG = os.environ.get("RRL_BUILD_TAG", "")
+BUILD = os.path.join(ROOT, "build", "rrl" + (f"-{_TAG}" if _TAG else ""))
 LIBDIR = os.path.join(HERE, "_lib")
-LIB = os.path.join(LIBDIR, "librrl.so")
+LIB = os.path.join(LIBDIR, "librrl" + (f"-{_TAG}" if _TAG else "") + ".so")
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
-COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", f"-I{INCLUDE}", f"-I{CSRC}"]
+COMMON = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", f"-I{INCLUDE}", f"-I{CSRC}",
+          *os.environ.get("RRL_NVCC_EXTRA", "").split()]
 
 
 def sources() -> list[str]:

@@ -752,6 +752,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       d.out = buffer_ptr(I, o.dest);
       d.buf1 = (o.child1 >= I->n_tips) ? o.child1 - I->n_tips : -1;
       d.buf2 = (o.child2 >= I->n_tips) ? o.child2 - I->n_tips : -1;
+      d.bufd = o.dest - I->n_tips;
       d.mat1 = o.matrix1;
       d.mat2 = o.matrix2;
       d.pat0 = ranges ? ranges[2 * i] : 0;

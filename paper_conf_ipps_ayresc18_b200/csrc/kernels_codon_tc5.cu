@@ -30,7 +30,8 @@
 //    four accumulators (tcgen05.ld 32x32b.x16), releases `acc_empty`, parks
 //    child 1 in the category's TMEM slot, forms the product with child 2, parks
 //    it in the same slot until the tile's last category, then scales by 2^-e
-//    and writes every category once, coalesced, through a swizzled staging tile.
+//    and writes every category once through a swizzled staging tile that a TMA
+//    bulk tensor store drains asynchronously (padding rows as zeros).
 // Compared with K3-TC (kernels_codon_tc.cu) the SM no longer moves the child
 // tile through registers: per phase it only writes the lo halves.
 #include <cuda.h>
@@ -41,6 +42,20 @@
 #include "rrl_internal.h"
 
 namespace rrl {
+
+#ifdef RRL_TC5_TRACE  // dev build only (tools/trace_tc5.py): clock64 timeline of CTA 0
+__device__ long long g_tc5_trace[12][4096];
+__device__ int g_tc5_kind[4096];
+#define TR(ev, g)                                                            \
+  do {                                                                       \
+    if (blockIdx.x == 0 && (g) < 4096) g_tc5_trace[ev][g] = clock64();      \
+  } while (0)
+#else
+#define TR(ev, g) \
+  do {            \
+  } while (0)
+#endif
+
 namespace {
 
 constexpr int TM = 128;  // patterns per tile = MMA M = TMEM lanes
@@ -105,6 +120,14 @@ __device__ inline void tma4(uint32_t dst, const void *tmap, int x, int y, int z,
       "l"(tmap), "r"(x), "r"(y), "r"(z), "r"(w), "r"(sa(bar))
       : "memory");
 }
+__device__ inline void tma_store4(const void *tmap, int x, int y, int z, int w, uint32_t src) {
+  asm volatile("cp.async.bulk.tensor.4d.global.shared::cta.bulk_group [%0, {%1, %2, %3, %4}], [%5];" ::"l"(tmap),
+               "r"(x), "r"(y), "r"(z), "r"(w), "r"(src)
+               : "memory");
+}
+__device__ inline void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
+__device__ inline void bulk_wait_read0() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ inline void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ inline void tmem_ld16(uint32_t taddr, float (&v)[16]) {
   uint32_t r[16];
   asm volatile(
@@ -202,6 +225,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
         const int buf = b == 0 ? op.buf1 : op.buf2, mat = b == 0 ? op.mat1 : op.mat2;
         bar_wait(&empty[s], ((uint32_t)(g >> 1) & 1u) ^ 1u);  // MMAs of phase g-2 are done
+        TR(0, g);
+#ifdef RRL_TC5_TRACE
+        if (blockIdx.x == 0 && g < 4096) g_tc5_kind[g] = tip ? 1 : 0;
+#endif
         const uint32_t st = sbase + s * ST_BYTES;
         bar_expect(&tma_full[s], (tip ? 0u : 32768u + 16384u) + 16384u);
         if (!tip) {  // child tile + the matrix's precomputed tf32 low parts (written by K1)
@@ -227,6 +254,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         bar_wait(acc_empty, (ni & 1u) ^ 1u);  // the epilogue drained the previous accumulators
         ++ni;
         fence_after();
+        TR(3, g);
         const uint32_t st = sbase + s * ST_BYTES;
         // per K-step of 8: A_hi . [P_hi | P_lo]^T (N = 128) -> [main_h | corr_h], then
         // A_lo . P_hi^T (N = 64) -> corr_h; main and the ~2^-11-smaller corrections
@@ -243,6 +271,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         }
         commit(&empty[s]);  // stage free once these MMAs completed
         commit(acc_full);   // accumulators ready for the epilogue
+        TR(4, g);
       }
     }
   } else if (warp >= kEpiThr / 32) {
@@ -254,6 +283,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
       unsigned char *st = sm + s * ST_BYTES;
       bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
+      if (ct == 0) TR(1, g);
       if (!tip) {  // a tip phase only lands P for the epilogue's gather: nothing to convert
 #pragma unroll
         for (int u = 0; u < TM * 16 / kConvThr; u += 8) {  // lo of every 16-byte chunk, same swizzled offset
@@ -268,6 +298,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
       __syncwarp();
+      if (ct == 0) TR(2, g);
       if (lane == 0) bar_arrive(&conv_full[s]);
     }
   } else {
@@ -275,9 +306,32 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     const int h = warp >> 2;               // column half
     const int r = (warp & 3) * 32 + lane;  // TMEM lane = pattern row of the tile
     const uint32_t tl = tmem + ((uint32_t)((warp & 3) * 32) << 16) + (uint32_t)(h * 32);
-    auto s1 = [&](int row, int k) -> float4 * {  // 16 x 16-byte chunks per row, chunk k at k ^ (row & 15)
-      return reinterpret_cast<float4 *>(S1 + row * TS + 4 * (k ^ (row & 15)));
+    // output staging in the TMA store's SWIZZLE_128B layout: column half hh is a
+    // 16 KB box of 128 rows x 128 B, 16-byte chunk j of row `row` at j ^ (row & 7)
+    auto s1 = [&](int row, int hh, int j) -> float4 * {
+      return reinterpret_cast<float4 *>(S1 + hh * (TM * 32) + row * 32 + 4 * (j ^ (row & 7)));
     };
+    // Row metadata of a tile (tip states of both children, the children's summed
+    // cumulative exponents or the stored factor to apply), loaded one tile ahead so
+    // the global-memory latency hides behind the current tile's phases.
+    auto load_meta = [&](int lt, uint32_t &sv, int &ex) {
+      const int f = blockIdx.x + lt * gridDim.x;
+      const DevOp &op = ops[f / ntiles];
+      const int pp = (f % ntiles) * TM + r;
+      const bool valid = pp < op.p;
+      const uint32_t s1v = (valid && (op.flags & OP_TIP1)) ? static_cast<const uint8_t *>(op.in1)[pp] : 0u;
+      const uint32_t s2v = (valid && (op.flags & OP_TIP2)) ? static_cast<const uint8_t *>(op.in2)[pp] : 0u;
+      sv = s1v | (s2v << 8);
+      ex = 0;
+      if (valid && op.scale_out != nullptr) {
+        if (op.cum1 != nullptr) ex += op.cum1[pp];
+        if (op.cum2 != nullptr) ex += op.cum2[pp];
+      } else if (valid && op.scale_in != nullptr) {
+        ex = op.scale_in[pp];
+      }
+    };
+    uint32_t sv_cur = 0, sv_nxt = 0;
+    int ex_cur = 0, ex_nxt = 0;
     float m = 0.f;  // running max over (c, z) of this thread's row half
     uint32_t ni = 0;  // internal-child phases consumed (accumulator barrier parity)
     for (int g = 0; g < nphase; ++g) {
@@ -287,6 +341,12 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       const int p0 = (f % ntiles) * TM;
       const int pp = p0 + r;
       const bool valid = pp < op.p;
+      if (c == 0 && b == 0) {  // tile start: rotate the prefetched metadata
+        if (lt == 0) load_meta(0, sv_nxt, ex_nxt);
+        sv_cur = sv_nxt;
+        ex_cur = ex_nxt;
+        if (lt + 1 < my_tiles) load_meta(lt + 1, sv_nxt, ex_nxt);
+      }
       float dv[32];
       if (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) {
         // Tip child: sum_x P[z][x] [x == obs] = P[z][obs], read from the raw fp32 P tile the
@@ -294,9 +354,9 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         // position chunk ^ (z&7) of half x>>5). A missing state (code >= 61) is the row sum.
         const int s = g & 1;
         bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
+        if (tid == 0) TR(7, g);
         const unsigned char *pt = sm + s * ST_BYTES + ST_B;  // P hi of K-half h at h * 16 KB
-        const uint8_t *states = static_cast<const uint8_t *>(b == 0 ? op.in1 : op.in2);  // range-offset
-        const unsigned sv = valid ? (unsigned)states[pp] : 0u;
+        const unsigned sv = (sv_cur >> (8 * b)) & 0xffu;  // prefetched (0 for padding rows)
         if (sv < (unsigned)kS61) {
           const unsigned char *base = pt + (sv >> 5) * 16384 + (sv & 3) * 4;
           const unsigned j = (sv & 31) >> 2;
@@ -321,10 +381,13 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         }
         named_sync(1, kEpiThr);  // every epilogue thread has read the P tile
         if (tid == 0) bar_arrive(&empty[s]);
+        if (tid == 0) TR(5, g);
       } else {
+        if (tid == 0) TR(11, g);
         bar_wait(acc_full, ni & 1u);
         ++ni;
         fence_after();
+        if (tid == 0) TR(7, g);
 #pragma unroll
         for (int q = 0; q < 2; ++q) {
           float m0[16], c0[16], m1[16], c1[16];
@@ -339,12 +402,14 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         fence_before();
         __syncwarp();
         if (lane == 0) bar_arrive(acc_empty);  // the MMAs of the next internal phase may overwrite them
+        if (tid == 0) TR(5, g);
       }
       const uint32_t slot = tl + (uint32_t)(kProdCol + c * TS);  // this category's TMEM slot
       if (b == 0) {  // child 1 waits in the slot until child 2's phase
         tmem_st16(slot, dv);
         tmem_st16(slot + 16, dv + 16);
         tmem_wait_st();
+        if (tid == 0) TR(6, g);
         continue;
       }
       {
@@ -364,6 +429,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         tmem_st16(slot, dv);
         tmem_st16(slot + 16, dv + 16);
         tmem_wait_st();
+        if (tid == 0) TR(6, g);
         continue;
       }
       // ---- tile done: row exponent from max over (c, z) of both column halves
@@ -374,20 +440,15 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         int e = 0;
         if (op.scale_out != nullptr) {
           e = frexp_e(mm);
-          if (valid) {
-            int tot = e;
-            if (op.cum1 != nullptr) tot += op.cum1[pp];
-            if (op.cum2 != nullptr) tot += op.cum2[pp];
-            op.scale_out[pp] = tot;
-          }
+          if (valid) op.scale_out[pp] = e + ex_cur;  // + the children's cumulative exponents
         } else if (op.scale_in != nullptr) {
-          e = valid ? op.scale_in[pp] : 0;
+          e = ex_cur;  // stored factor (0 for padding rows)
         }
         mx[r] = (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
       }
       named_sync(1, kEpiThr);
+      if (tid == 0) TR(8, g);
       const float sc = mx[r];
-      float *out = static_cast<float *>(op.out);
       for (int cat = 0; cat < C; ++cat) {
         float v[32];
         if (cat < C - 1) {
@@ -401,21 +462,27 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
 #pragma unroll
           for (int i = 0; i < 32; ++i) v[i] = dv[i];
         }
-        named_sync(1, kEpiThr);  // staging tile free
-#pragma unroll
-        for (int k = 0; k < 8; ++k)
-          *s1(r, h * 8 + k) = make_float4(v[4 * k] * sc, v[4 * k + 1] * sc, v[4 * k + 2] * sc, v[4 * k + 3] * sc);
+        if (tid == 0) bulk_wait_read0();  // the previous TMA store has read the staging tile
         named_sync(1, kEpiThr);
 #pragma unroll
-        for (int u = 0; u < TM * 16 / kEpiThr; ++u) {  // coalesced: a warp writes 2 rows
-          const int i = tid + u * kEpiThr, row = i >> 4, ch = i & 15;
-          if (p0 + row < op.p)
-            *reinterpret_cast<float4 *>(out + ((size_t)cat * p_pad + p0 + row) * TS + ch * 4) = *s1(row, ch);
+        for (int k = 0; k < 8; ++k)
+          *s1(r, h, k) = valid ? make_float4(v[4 * k] * sc, v[4 * k + 1] * sc, v[4 * k + 2] * sc, v[4 * k + 3] * sc)
+                               : make_float4(0.f, 0.f, 0.f, 0.f);  // padding rows of the tile: zeros
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> TMA store
+        named_sync(1, kEpiThr);
+        if (tid == 0) {  // asynchronous: the tile's HBM writes overlap the next tile's phases
+          tma_store4(&tmA, 0, op.pat0 + p0, cat, op.bufd, sa(S1));
+          tma_store4(&tmA, 32, op.pat0 + p0, cat, op.bufd, sa(S1) + TM * 128);
+          bulk_commit();
+          if (cat == 0) TR(9, g);
+          if (cat == C - 1) TR(10, g);
         }
       }
+      if (tid == 0) TR(6, g);
       m = 0.f;  // (the next tile's first staging write waits at the loop's first barrier)
     }
   }
+  if (tid == 0) bulk_wait0();  // output stores complete before the grid does
   fence_before();
   __syncthreads();
   if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
@@ -456,9 +523,11 @@ int launch_tc5(const DevOp *d_ops, int nops, int p, int p_pad, const CUtensorMap
 int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
                                      int p_pad, const void *tmap_partials, const void *tmap_P,
                                      const void *tmap_Plo, void *stream) {
-  // every child must live in the tensor-mapped slab (internal buffers) or be tip states
+  // every child must live in the tensor-mapped slab (internal buffers) or be tip states; the
+  // destination is always in the slab (its tile is written back by TMA store)
   for (int i = 0; i < nops; ++i)
-    if ((!(h_ops[i].flags & OP_TIP1) && h_ops[i].buf1 < 0) || (!(h_ops[i].flags & OP_TIP2) && h_ops[i].buf2 < 0))
+    if ((!(h_ops[i].flags & OP_TIP1) && h_ops[i].buf1 < 0) || (!(h_ops[i].flags & OP_TIP2) && h_ops[i].buf2 < 0) ||
+        h_ops[i].bufd < 0)
       return (int)cudaErrorNotSupported;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   const CUtensorMap *tA = static_cast<const CUtensorMap *>(tmap_partials);
@@ -473,3 +542,11 @@ int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_o
 }
 
 }  // namespace rrl
+
+#ifdef RRL_TC5_TRACE
+extern "C" int rrl_debug_tc5_trace(long long *ev /*[12*4096]*/, int *kind /*[4096]*/) {
+  if (cudaMemcpyFromSymbol(ev, rrl::g_tc5_trace, sizeof(rrl::g_tc5_trace)) != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(kind, rrl::g_tc5_kind, sizeof(rrl::g_tc5_kind)) != cudaSuccess) return -1;
+  return 0;
+}
+#endif

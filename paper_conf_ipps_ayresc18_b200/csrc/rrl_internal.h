@@ -31,7 +31,7 @@ struct DevOp {
   int32_t buf1, buf2;       // child internal-buffer index in the partials slab, -1 if not in it
   int32_t mat1, mat2;       // transition-matrix indices
   int32_t pat0;             // first pattern of the range
-  int32_t pad_;
+  int32_t bufd;             // dest internal-buffer index in the partials slab
 };
 static_assert(sizeof(DevOp) == 104, "DevOp layout");
 

@@ -13,7 +13,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "_lib", "librrl.so")
+LIB_PATH = os.environ.get("RRL_LIB_PATH") or os.path.join(_HERE, "_lib", "librrl.so")  # override: dev builds
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} not built: run `python -m paper_conf_ipps_ayresc18_b200.build`"
