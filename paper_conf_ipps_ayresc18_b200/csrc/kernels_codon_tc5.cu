@@ -63,16 +63,17 @@ constexpr int TS = 64;   // padded states: MMA N and K
 constexpr int kS61 = 61;
 constexpr int kEpiThr = 256;                 // warps 0-7
 constexpr int kConvThr = 128;                // warps 8-11
-constexpr int kProdWarp = 12, kMmaWarp = 13;
-constexpr int kThr = 14 * 32;
-// one stage: A hi (2 x 16 KB halves k 0-31 / 32-63), A lo, then B = per K-half h
-// [P hi rows 0-63 | P lo rows 0-63] (16 KB), so one N = 128 MMA reads A hi once
-// for both hi.hi and hi.lo.
-constexpr int ST_AHI = 0, ST_ALO = 32768, ST_B = 65536, ST_BYTES = 98304;
-constexpr int SMEM_S1 = 2 * ST_BYTES;                  // epilogue staging tile (32 KB)
-constexpr int SMEM_MX = SMEM_S1 + TM * TS * 4;         // row maxima / scale [2][128]
-constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 8 mbarriers
-constexpr int SMEM_TMEM = SMEM_BAR + 8 * 8;
+constexpr int kProdA = 12, kMmaWarp = 13, kProdB = 14;
+constexpr int kThr = 15 * 32;
+// Shared memory: a ring of NA raw child tiles (TMA; the tf32 hi operand, two
+// 16 KB K-halves each), one tile of lo parts, a ring of two matrix tiles (per
+// K-half h: [P hi rows 0-63 | P lo rows 0-63], 16 KB, so one N = 128 MMA reads
+// A hi once for hi.hi and hi.lo), the output staging tile.
+constexpr int NA = 3, NB = 2;
+constexpr int SM_A = 0, SM_ALO = NA * 32768, SM_B = SM_ALO + 32768, SM_S1 = SM_B + NB * 32768;
+constexpr int SMEM_MX = SM_S1 + TM * TS * 4;           // row maxima / scale [2][128]
+constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 16 mbarriers
+constexpr int SMEM_TMEM = SMEM_BAR + 16 * 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 16;
 constexpr int kTmemCols = 512;    // per K-half h: [main_h | corr_h] (4 x 64) ...
 constexpr int kProdCol = 4 * TS;  // ... + one 64-column slot per category (child 1, then the product)
@@ -174,13 +175,16 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
                      const __grid_constant__ CUtensorMap tmPlo) {
   static_assert(kProdCol + C * TS <= kTmemCols, "category slots must fit TMEM");
   extern __shared__ __align__(1024) unsigned char sm[];
-  uint64_t *tma_full = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);  // [2]
-  uint64_t *conv_full = tma_full + 2;                                 // [2]
-  uint64_t *empty = tma_full + 4;                                     // [2]
-  uint64_t *acc_full = tma_full + 6;
-  uint64_t *acc_empty = tma_full + 7;
+  uint64_t *a_full = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);  // [NA] child tile landed
+  uint64_t *a_empty = a_full + NA;                                  // [NA] its MMAs completed
+  uint64_t *b_full = a_full + 2 * NA;                               // [NB] matrix tile landed
+  uint64_t *b_empty = b_full + NB;                                  // [NB] MMAs / tip gather done
+  uint64_t *lo_full = b_full + 2 * NB;                              // converters wrote the lo tile
+  uint64_t *lo_empty = lo_full + 1;                                 // its MMAs completed
+  uint64_t *acc_full = lo_full + 2;
+  uint64_t *acc_empty = lo_full + 3;
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(sm + SMEM_TMEM);
-  float *S1 = reinterpret_cast<float *>(sm + SMEM_S1);
+  float *S1 = reinterpret_cast<float *>(sm + SM_S1);
   float *mx = reinterpret_cast<float *>(sm + SMEM_MX);
   const uint32_t sbase = sa(sm);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -191,12 +195,17 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
                  "r"(kTmemCols));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
-  if (tid == kProdWarp * 32) {
-    for (int s = 0; s < 2; ++s) {
-      bar_init(&tma_full[s], 1);
-      bar_init(&conv_full[s], kConvThr / 32);
-      bar_init(&empty[s], 1);
+  if (tid == kProdA * 32) {
+    for (int i = 0; i < NA; ++i) {
+      bar_init(&a_full[i], 1);
+      bar_init(&a_empty[i], 1);
     }
+    for (int i = 0; i < NB; ++i) {
+      bar_init(&b_full[i], 1);
+      bar_init(&b_empty[i], 1);
+    }
+    bar_init(lo_full, kConvThr / 32);
+    bar_init(lo_empty, 1);
     bar_init(acc_full, 1);
     bar_init(acc_empty, kEpiThr / 32);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -214,92 +223,125 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
   const int my_tiles = total > (int)blockIdx.x ? (total - 1 - (int)blockIdx.x) / (int)gridDim.x + 1 : 0;
   const int nphase = my_tiles * C * 2;  // (tile, category, child)
 
-  if (warp == kProdWarp) {
-    // ================================================================ TMA producer
+  // phase g = (local tile lt, category c, child b); internal-child phases are
+  // counted separately (ia): only they use the child-tile ring and the lo tile.
+  auto phase_op = [&](int g, int &c, int &b, int &p0) -> const DevOp & {
+    const int lt = g / (2 * C), f = blockIdx.x + lt * gridDim.x;
+    c = (g / 2) % C;
+    b = g & 1;
+    p0 = (f % ntiles) * TM;
+    return ops[f / ntiles];
+  };
+  auto is_tip = [](const DevOp &op, int b) { return (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0; };
+
+  if (warp == kProdA) {
+    // ================================================================ child-tile producer
+    if (lane == 0) {
+      uint32_t ia = 0;
+      for (int g = 0; g < nphase; ++g) {
+        int c, b, p0;
+        const DevOp &op = phase_op(g, c, b, p0);
+        if (is_tip(op, b)) continue;
+        const uint32_t sl = ia % NA, use = ia / NA;
+        ++ia;
+        bar_wait(&a_empty[sl], (use & 1u) ^ 1u);  // the MMAs NA internal phases back are done
+        TR(0, g);
+        const uint32_t dst = sbase + SM_A + sl * 32768;
+        bar_expect(&a_full[sl], 32768u);
+        const int buf = b == 0 ? op.buf1 : op.buf2;
+        tma4(dst, &tmA, 0, op.pat0 + p0, c, buf, &a_full[sl]);
+        tma4(dst + 16384, &tmA, 32, op.pat0 + p0, c, buf, &a_full[sl]);
+      }
+    }
+  } else if (warp == kProdB) {
+    // ================================================================ matrix producer
     if (lane == 0) {
       for (int g = 0; g < nphase; ++g) {
-        const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1, s = g & 1;
-        const int f = blockIdx.x + lt * gridDim.x;
-        const DevOp &op = ops[f / ntiles];
-        const int p0 = (f % ntiles) * TM;
-        const bool tip = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
-        const int buf = b == 0 ? op.buf1 : op.buf2, mat = b == 0 ? op.mat1 : op.mat2;
-        bar_wait(&empty[s], ((uint32_t)(g >> 1) & 1u) ^ 1u);  // MMAs of phase g-2 are done
-        TR(0, g);
+        int c, b, p0;
+        const DevOp &op = phase_op(g, c, b, p0);
+        const bool tip = is_tip(op, b);
+        const uint32_t sl = g % NB, use = g / NB;
+        bar_wait(&b_empty[sl], (use & 1u) ^ 1u);
 #ifdef RRL_TC5_TRACE
         if (blockIdx.x == 0 && g < 4096) g_tc5_kind[g] = tip ? 1 : 0;
 #endif
-        const uint32_t st = sbase + s * ST_BYTES;
-        bar_expect(&tma_full[s], (tip ? 0u : 32768u + 16384u) + 16384u);
-        if (!tip) {  // child tile + the matrix's precomputed tf32 low parts (written by K1)
-          tma4(st + ST_AHI, &tmA, 0, op.pat0 + p0, c, buf, &tma_full[s]);
-          tma4(st + ST_AHI + 16384, &tmA, 32, op.pat0 + p0, c, buf, &tma_full[s]);
-          tma4(st + ST_B + 8192, &tmPlo, 0, 0, c, mat, &tma_full[s]);
-          tma4(st + ST_B + 16384 + 8192, &tmPlo, 32, 0, c, mat, &tma_full[s]);
+        const uint32_t dst = sbase + SM_B + sl * 32768;
+        const int mat = b == 0 ? op.mat1 : op.mat2;
+        bar_expect(&b_full[sl], tip ? 16384u : 32768u);
+        tma4(dst, &tmP, 0, 0, c, mat, &b_full[sl]);
+        tma4(dst + 16384, &tmP, 32, 0, c, mat, &b_full[sl]);
+        if (!tip) {  // the matrix's tf32 low parts, precomputed by K1
+          tma4(dst + 8192, &tmPlo, 0, 0, c, mat, &b_full[sl]);
+          tma4(dst + 16384 + 8192, &tmPlo, 32, 0, c, mat, &b_full[sl]);
         }
-        tma4(st + ST_B, &tmP, 0, 0, c, mat, &tma_full[s]);
-        tma4(st + ST_B + 16384, &tmP, 32, 0, c, mat, &tma_full[s]);
       }
     }
   } else if (warp == kMmaWarp) {
     // ================================================================ MMA issuer
     if (lane == 0) {
-      uint32_t ni = 0;  // internal-child phases issued (accumulator barrier parity)
+      uint32_t ia = 0;
       for (int g = 0; g < nphase; ++g) {
-        const int lt = g / (2 * C), b = g & 1, s = g & 1;
-        const int f = blockIdx.x + lt * gridDim.x;
-        const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
-        bar_wait(&conv_full[s], (uint32_t)(g >> 1) & 1u);
-        if (tip) continue;  // a tip child is a P-column gather in the epilogue: no MMA
-        bar_wait(acc_empty, (ni & 1u) ^ 1u);  // the epilogue drained the previous accumulators
-        ++ni;
+        int c, b, p0;
+        const DevOp &op = phase_op(g, c, b, p0);
+        const uint32_t bs = g % NB;
+        bar_wait(&b_full[bs], (uint32_t)(g / NB) & 1u);
+        if (is_tip(op, b)) continue;  // a tip child is a P-column gather in the epilogue: no MMA
+        const uint32_t sl = ia % NA, use = ia / NA;
+        bar_wait(&a_full[sl], use & 1u);
+        bar_wait(lo_full, ia & 1u);
+        bar_wait(acc_empty, (ia & 1u) ^ 1u);  // the epilogue drained the previous accumulators
+        ++ia;
         fence_after();
         TR(3, g);
-        const uint32_t st = sbase + s * ST_BYTES;
         // per K-step of 8: A_hi . [P_hi | P_lo]^T (N = 128) -> [main_h | corr_h], then
         // A_lo . P_hi^T (N = 64) -> corr_h; main and the ~2^-11-smaller corrections
         // never share an accumulator (tf32 accumulation reading).
 #pragma unroll
         for (int kk = 0; kk < TS / 8; ++kk) {
           const int h = kk >> 2, kin = kk & 3;
-          const uint64_t ah = desc_sw128(st + ST_AHI + h * 16384 + kin * 32);
-          const uint64_t al = desc_sw128(st + ST_ALO + h * 16384 + kin * 32);
-          const uint64_t bb = desc_sw128(st + ST_B + h * 16384 + kin * 32);
+          const uint64_t ah = desc_sw128(sbase + SM_A + sl * 32768 + h * 16384 + kin * 32);
+          const uint64_t al = desc_sw128(sbase + SM_ALO + h * 16384 + kin * 32);
+          const uint64_t bb = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + kin * 32);
           const uint32_t d = tmem + (uint32_t)(h * 2 * TS);
           mma_tf32(d, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);
           mma_tf32(d + TS, al, bb, idesc_tf32(TS), 1u);
         }
-        commit(&empty[s]);  // stage free once these MMAs completed
-        commit(acc_full);   // accumulators ready for the epilogue
+        commit(&a_empty[sl]);  // child tile, lo tile and matrix tile free once these MMAs completed
+        commit(lo_empty);
+        commit(&b_empty[bs]);
+        commit(acc_full);  // accumulators ready for the epilogue
         TR(4, g);
       }
     }
-  } else if (warp >= kEpiThr / 32) {
+  } else if (warp >= kEpiThr / 32 && warp < kEpiThr / 32 + kConvThr / 32) {
     // ================================================================ converters
     const int ct = tid - kEpiThr;
+    uint32_t ia = 0;
     for (int g = 0; g < nphase; ++g) {
-      const int lt = g / (2 * C), b = g & 1, s = g & 1;
-      const int f = blockIdx.x + lt * gridDim.x;
-      const bool tip = (ops[f / ntiles].flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
-      unsigned char *st = sm + s * ST_BYTES;
-      bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
+      int c, b, p0;
+      const DevOp &op = phase_op(g, c, b, p0);
+      if (is_tip(op, b)) continue;
+      const uint32_t sl = ia % NA, use = ia / NA;
+      bar_wait(&a_full[sl], use & 1u);
+      bar_wait(lo_empty, (ia & 1u) ^ 1u);  // the previous internal phase's MMAs read the lo tile
+      ++ia;
       if (ct == 0) TR(1, g);
-      if (!tip) {  // a tip phase only lands P for the epilogue's gather: nothing to convert
+      const unsigned char *src = sm + SM_A + sl * 32768;
+      unsigned char *dst = sm + SM_ALO;
 #pragma unroll
-        for (int u = 0; u < TM * 16 / kConvThr; u += 8) {  // lo of every 16-byte chunk, same swizzled offset
-          float4 v[8];
+      for (int u = 0; u < TM * 16 / kConvThr; u += 8) {  // lo of every 16-byte chunk, same swizzled offset
+        float4 v[8];
 #pragma unroll
-          for (int q = 0; q < 8; ++q) v[q] = *reinterpret_cast<const float4 *>(st + ST_AHI + (ct + (u + q) * kConvThr) * 16);
+        for (int q = 0; q < 8; ++q) v[q] = *reinterpret_cast<const float4 *>(src + (ct + (u + q) * kConvThr) * 16);
 #pragma unroll
-          for (int q = 0; q < 8; ++q)
-            *reinterpret_cast<float4 *>(st + ST_ALO + (ct + (u + q) * kConvThr) * 16) =
-                make_float4(lo_tf32(v[q].x), lo_tf32(v[q].y), lo_tf32(v[q].z), lo_tf32(v[q].w));
-        }
+        for (int q = 0; q < 8; ++q)
+          *reinterpret_cast<float4 *>(dst + (ct + (u + q) * kConvThr) * 16) =
+              make_float4(lo_tf32(v[q].x), lo_tf32(v[q].y), lo_tf32(v[q].z), lo_tf32(v[q].w));
       }
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
       __syncwarp();
       if (ct == 0) TR(2, g);
-      if (lane == 0) bar_arrive(&conv_full[s]);
+      if (lane == 0) bar_arrive(lo_full);
     }
   } else {
     // ================================================================ epilogue
@@ -352,10 +394,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         // Tip child: sum_x P[z][x] [x == obs] = P[z][obs], read from the raw fp32 P tile the
         // producer landed in stage g&1 (swizzled K-major: row z, 16-byte chunk (x&31)/4 at
         // position chunk ^ (z&7) of half x>>5). A missing state (code >= 61) is the row sum.
-        const int s = g & 1;
-        bar_wait(&tma_full[s], (uint32_t)(g >> 1) & 1u);
+        const int s = g % NB;
+        bar_wait(&b_full[s], (uint32_t)(g / NB) & 1u);
         if (tid == 0) TR(7, g);
-        const unsigned char *pt = sm + s * ST_BYTES + ST_B;  // P hi of K-half h at h * 16 KB
+        const unsigned char *pt = sm + SM_B + s * 32768;  // P hi of K-half h at h * 16 KB
         const unsigned sv = (sv_cur >> (8 * b)) & 0xffu;  // prefetched (0 for padding rows)
         if (sv < (unsigned)kS61) {
           const unsigned char *base = pt + (sv >> 5) * 16384 + (sv & 3) * 4;
@@ -380,7 +422,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
           }
         }
         named_sync(1, kEpiThr);  // every epilogue thread has read the P tile
-        if (tid == 0) bar_arrive(&empty[s]);
+        if (tid == 0) bar_arrive(&b_empty[s]);
         if (tid == 0) TR(5, g);
       } else {
         if (tid == 0) TR(11, g);
