@@ -374,6 +374,33 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     };
     uint32_t sv_cur = 0, sv_nxt = 0;
     int ex_cur = 0, ex_nxt = 0;
+    // write-back of the previous tile: scale slot `cat` by 2^-e, stage it in the
+    // swizzled layout, and hand it to an asynchronous TMA bulk tensor store
+    float sc_prev = 0.f;
+    int prev_y = 0, prev_buf = 0;
+    bool have_prev = false;
+    auto drain = [&](int cat) {
+      float w0[16], w1[16];
+      tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), w0);
+      tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), w1);
+      tmem_wait_ld();
+      if (tid == 0) bulk_wait_read0();  // the previous store has read the staging tile
+      named_sync(1, kEpiThr);
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        *s1(r, h, k) = make_float4(w0[4 * k] * sc_prev, w0[4 * k + 1] * sc_prev, w0[4 * k + 2] * sc_prev,
+                                   w0[4 * k + 3] * sc_prev);
+        *s1(r, h, 4 + k) = make_float4(w1[4 * k] * sc_prev, w1[4 * k + 1] * sc_prev, w1[4 * k + 2] * sc_prev,
+                                       w1[4 * k + 3] * sc_prev);
+      }
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> TMA store
+      named_sync(1, kEpiThr);
+      if (tid == 0) {
+        tma_store4(&tmA, 0, prev_y, cat, prev_buf, sa(S1));
+        tma_store4(&tmA, 32, prev_y, cat, prev_buf, sa(S1) + TM * 128);
+        bulk_commit();
+      }
+    };
     float m = 0.f;  // running max over (c, z) of this thread's row half
     uint32_t ni = 0;  // internal-child phases consumed (accumulator barrier parity)
     for (int g = 0; g < nphase; ++g) {
@@ -383,6 +410,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       const int p0 = (f % ntiles) * TM;
       const int pp = p0 + r;
       const bool valid = pp < op.p;
+      if (b == 0 && have_prev) {  // before child 1 reuses slot c: write back the previous tile's category c
+        drain(c);
+        if (tid == 0) TR(9, g);
+      }
       if (c == 0 && b == 0) {  // tile start: rotate the prefetched metadata
         if (lt == 0) load_meta(0, sv_nxt, ex_nxt);
         sv_cur = sv_nxt;
@@ -467,10 +498,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
 #pragma unroll
         for (int i = 0; i < 32; ++i) m = fmaxf(m, dv[i]);
       }
-      if (c < C - 1) {  // park the unscaled product (in place of child 1) until the tile's exponent is known
-        tmem_st16(slot, dv);
-        tmem_st16(slot + 16, dv + 16);
-        tmem_wait_st();
+      tmem_st16(slot, dv);  // park the unscaled product (in place of child 1) until written back
+      tmem_st16(slot + 16, dv + 16);
+      tmem_wait_st();
+      if (c < C - 1) {
         if (tid == 0) TR(6, g);
         continue;
       }
@@ -490,39 +521,17 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       }
       named_sync(1, kEpiThr);
       if (tid == 0) TR(8, g);
-      const float sc = mx[r];
-      for (int cat = 0; cat < C; ++cat) {
-        float v[32];
-        if (cat < C - 1) {
-          float lo16[16], hi16[16];
-          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), lo16);
-          tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), hi16);
-          tmem_wait_ld();
-#pragma unroll
-          for (int i = 0; i < 16; ++i) { v[i] = lo16[i]; v[16 + i] = hi16[i]; }
-        } else {
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = dv[i];
-        }
-        if (tid == 0) bulk_wait_read0();  // the previous TMA store has read the staging tile
-        named_sync(1, kEpiThr);
-#pragma unroll
-        for (int k = 0; k < 8; ++k)
-          *s1(r, h, k) = valid ? make_float4(v[4 * k] * sc, v[4 * k + 1] * sc, v[4 * k + 2] * sc, v[4 * k + 3] * sc)
-                               : make_float4(0.f, 0.f, 0.f, 0.f);  // padding rows of the tile: zeros
-        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> TMA store
-        named_sync(1, kEpiThr);
-        if (tid == 0) {  // asynchronous: the tile's HBM writes overlap the next tile's phases
-          tma_store4(&tmA, 0, op.pat0 + p0, cat, op.bufd, sa(S1));
-          tma_store4(&tmA, 32, op.pat0 + p0, cat, op.bufd, sa(S1) + TM * 128);
-          bulk_commit();
-          if (cat == 0) TR(9, g);
-          if (cat == C - 1) TR(10, g);
-        }
-      }
+      // the products wait in their slots; tile t's category c is written back during
+      // tile t+1's phase (c, child 1), so the TMA stores overlap the next tile's work
+      sc_prev = valid ? mx[r] : 0.f;  // padding rows of the tile are written as zeros
+      prev_y = op.pat0 + p0;
+      prev_buf = op.bufd;
+      have_prev = true;
       if (tid == 0) TR(6, g);
-      m = 0.f;  // (the next tile's first staging write waits at the loop's first barrier)
+      m = 0.f;
     }
+    if (have_prev)  // the CTA's last tile
+      for (int cat = 0; cat < C; ++cat) drain(cat);
   }
   if (tid == 0) bulk_wait0();  // output stores complete before the grid does
   fence_before();
