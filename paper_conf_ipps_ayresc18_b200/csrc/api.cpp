@@ -804,8 +804,10 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       Timed tm(I, 0, !capturing);  // eager profiling: one event pair per set launch
       int e;
       if (I->s == 4) {
+        // tip states may be read before the PDL wait; the matrices too unless this
+        // launch directly follows K1 (k = 0: K1 or a host update may be its predecessor)
         e = launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax,
-                                       I->p_pad, I->stream);
+                                       I->p_pad, k > 0 ? 3 : 1, I->stream);
       } else {
         e = (int)cudaErrorNotSupported;
         if (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT) && I->tmaps_ok)  // TMA-fed tcgen05 (c <= 4)

@@ -201,9 +201,14 @@ __device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
     v[z] = fma(P[z * 4 + 3], L[3], fma(P[z * 4 + 2], L[2], fma(P[z * 4 + 1], L[1], P[z * 4] * L[0])));
 }
 
+// `early` (host-decided): bit 0 -- tip states may be read before griddepcontrol.wait
+// (only host copies write them); bit 1 -- so may the transition matrices (K1 is
+// not this launch's immediate predecessor, so it completed before the previous
+// level set passed its own wait).  Only the previous level set's partials and
+// exponents must wait.
 template <typename T, int C, int U>
 __global__ void __launch_bounds__(kThreads)
-k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
+k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int early) {
   const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
   const int cat = threadIdx.x % C;  // kThreads is a multiple of C
@@ -218,24 +223,41 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
   const unsigned nitems = (unsigned)op.p * C;  // this operation's pattern range
   (void)p;
 
-  pdl_wait();  // everything above overlaps the previous level set
-  pdl_launch();
-
   // fp32: each thread holds its category's rows in registers.  fp64: the rows
   // would cost 64 registers, so the block stages the tables in shared memory
   // (issued after this thread's first child loads, see below).
   constexpr bool kRegP = sizeof(T) == 4;
   __shared__ __align__(16) T sP[kRegP ? 1 : 2][kRegP ? 1 : C][kRegP ? 4 : kPTab];
   T P1[kRegP ? 16 : 1], P2[kRegP ? 16 : 1];
-  if constexpr (kRegP) {
+  auto load_rows = [&]() {
+    if constexpr (kRegP) {
 #pragma unroll
-    for (int k = 0; k < 16; k += 4) {
-      V4<T>::ld(P1g + k, *reinterpret_cast<T(*)[4]>(&P1[k]));
-      V4<T>::ld(P2g + k, *reinterpret_cast<T(*)[4]>(&P2[k]));
+      for (int k = 0; k < 16; k += 4) {
+        V4<T>::ld(P1g + k, *reinterpret_cast<T(*)[4]>(&P1[k]));
+        V4<T>::ld(P2g + k, *reinterpret_cast<T(*)[4]>(&P2[k]));
+      }
+    }
+  };
+  // first chunk's tip states (and rows) in flight while the previous level set finishes
+  unsigned s1p[U], s2p[U];
+  if (early & 1) {
+#pragma unroll
+    for (int j = 0; j < U; ++j) {
+      const unsigned item = (unsigned)blockIdx.x * (kThreads * U) + threadIdx.x + j * kThreads;
+      const bool valid = item < nitems && (int)blockIdx.x < nchunks;
+      s1p[j] = (tip1 && valid) ? (unsigned)__ldg(S1g + item / C) : 4u;
+      s2p[j] = (tip2 && valid) ? (unsigned)__ldg(S2g + item / C) : 4u;
     }
   }
+  if (early & 2) load_rows();
+
+  pdl_wait();  // everything above overlaps the previous level set
+  pdl_launch();
+
+  if (!(early & 2)) load_rows();
   bool tables = kRegP;
   for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
+    const bool pre = (early & 1) && chunk == (int)blockIdx.x;
     const unsigned base = (unsigned)chunk * (kThreads * U) + threadIdx.x;
     T L1[U][4], L2[U][4];
     unsigned s1[U], s2[U];
@@ -246,7 +268,7 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
       const bool valid = item < nitems;
       const unsigned pat = item / C;
       if (tip1) {
-        s1[j] = valid ? (unsigned)__ldg(S1g + pat) : 4u;
+        s1[j] = pre ? s1p[j] : valid ? (unsigned)__ldg(S1g + pat) : 4u;
       } else if (valid) {
         V4<T>::ld(L1g + (size_t)item * 4, L1[j]);
       } else {
@@ -254,7 +276,7 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks) {
         for (int z = 0; z < 4; ++z) L1[j][z] = T(0);
       }
       if (tip2) {
-        s2[j] = valid ? (unsigned)__ldg(S2g + pat) : 4u;
+        s2[j] = pre ? s2p[j] : valid ? (unsigned)__ldg(S2g + pat) : 4u;
       } else if (valid) {
         V4<T>::ld(L2g + (size_t)item * 4, L2[j]);
       } else {
@@ -545,7 +567,7 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
 
 // ============================================================ host launchers
 template <typename T, int C, int U>
-int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int gx_cap,
+int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int gx_cap, int early,
                      cudaStream_t st) {
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads * U - 1) / (kThreads * U));
@@ -569,7 +591,7 @@ int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, in
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U>, pack, p, nchunks);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U>, pack, p, nchunks, early);
     if (e != cudaSuccess) return (int)e;
   }
   return 0;
@@ -581,7 +603,7 @@ int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, in
 // per step): a launch this small is bound by its one dependent memory round
 // trip, so the widest single round wins.
 template <typename T, int C>
-int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
+int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int early, cudaStream_t st) {
   static int resident = -1;  // per template instance
   if (resident < 0) {
     int per_sm = 1, dev = 0, nsm = 148;
@@ -590,7 +612,7 @@ int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cuda
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     resident = (per_sm > 0 ? per_sm : 1) * nsm;
   }
-  return launch_latency_u<T, C, 1>(d_ops, h_ops, nops, p, resident, st);
+  return launch_latency_u<T, C, 1>(d_ops, h_ops, nops, p, resident, early, st);
 }
 
 template <typename T, int C>
@@ -635,18 +657,18 @@ int launch_bulk(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
 constexpr long long kBulkMinItems = 64LL * 1024;
 
 template <typename T, int C>
-int launch_t(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
+int launch_t(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int early, cudaStream_t st) {
   if ((long long)p * C >= kBulkMinItems) return launch_bulk<T, C>(d_ops, nops, p, st);
-  return launch_latency<T, C>(d_ops, h_ops, nops, p, st);
+  return launch_latency<T, C>(d_ops, h_ops, nops, p, early, st);
 }
 
 template <typename T>
-int dispatch_c(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p, cudaStream_t st) {
+int dispatch_c(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int early, cudaStream_t st) {
   switch (c) {
-    case 1: return launch_t<T, 1>(d_ops, h_ops, nops, p, st);
-    case 2: return launch_t<T, 2>(d_ops, h_ops, nops, p, st);
-    case 4: return launch_t<T, 4>(d_ops, h_ops, nops, p, st);
-    case 8: return launch_t<T, 8>(d_ops, h_ops, nops, p, st);
+    case 1: return launch_t<T, 1>(d_ops, h_ops, nops, p, early, st);
+    case 2: return launch_t<T, 2>(d_ops, h_ops, nops, p, early, st);
+    case 4: return launch_t<T, 4>(d_ops, h_ops, nops, p, early, st);
+    case 8: return launch_t<T, 8>(d_ops, h_ops, nops, p, early, st);
     default: return (int)cudaErrorInvalidValue;
   }
 }
@@ -654,10 +676,10 @@ int dispatch_c(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p, c
 }  // namespace
 
 int launch_update_partials_nuc(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
-                               int p, int /*p_pad*/, void *stream) {
+                               int p, int /*p_pad*/, int early, void *stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  return prec == 32 ? dispatch_c<float>(c, d_ops, h_ops, nops, p, st)
-                    : dispatch_c<double>(c, d_ops, h_ops, nops, p, st);
+  return prec == 32 ? dispatch_c<float>(c, d_ops, h_ops, nops, p, early, st)
+                    : dispatch_c<double>(c, d_ops, h_ops, nops, p, early, st);
 }
 
 }  // namespace rrl

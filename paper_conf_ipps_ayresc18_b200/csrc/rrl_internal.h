@@ -42,7 +42,7 @@ enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2 };
 // d_ops: descriptors in device memory; h_ops: the same descriptors on the host
 // (small sets are passed by value in the kernel parameters), may be null.
 int launch_update_partials_nuc(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
-                               int p, int p_pad, void *stream);
+                               int p, int p_pad, int early, void *stream);
 int launch_update_partials_codon(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
                                  int p, int p_pad, void *stream);
 // tcgen05 (tf32, 3xTF32) codon kernel: fp32, c in {1,2,4,8}; cudaErrorNotSupported otherwise.
