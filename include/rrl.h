@@ -158,6 +158,10 @@ int rrl_synchronize(int inst);
 /* --------------------------------------------------------------------- data
  * Tip data (reading A23).  Tip partials are category-independent [p][s]. */
 int rrl_set_tip_states(int inst, int tip, const int32_t *states /*[p]*/);
+/* Tips first_tip..first_tip+count-1 as uint8 codes (0..s-1, s = missing),
+ * rows of p bytes.  One host->device DMA (fast from pinned memory); the code
+ * range is validated on the device.  A code > s returns
+ * RRL_ERROR_OUT_OF_RANGE and leaves those tips all-missing. */
 int rrl_set_tip_states_u8(int inst, int first_tip, int count,
                           const uint8_t *states /*[count][p]*/);
 int rrl_set_tip_partials(int inst, int tip, const double *partials /*[p][s]*/);

@@ -62,6 +62,7 @@ struct Instance {
   double *d_block = nullptr;             // [nblocks]
   double *d_out = nullptr;               // scalar
   unsigned *d_count = nullptr;           // last-block-done ticket of K4/K6
+  unsigned *d_flag = nullptr;            // tip-state validation result
   double *h_out = nullptr;               // pinned scalar
   int nblocks = 0;
 
@@ -197,7 +198,7 @@ void destroy(Instance *I) {
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
                   I->d_catw,     I->d_freqs,  I->d_pw,   I->d_site,  I->d_block, I->d_out, I->d_count,
-                  I->d_midx,     I->d_t,      I->d_sidx, I->d_ops,  I->d_Plo};
+                  I->d_midx,     I->d_t,      I->d_sidx, I->d_ops,  I->d_Plo,  I->d_flag};
   for (void *q : ptrs)
     if (q) cudaFree(q);
   if (I->h_ops) cudaFreeHost(I->h_ops);
@@ -382,6 +383,7 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
     }
   }
   CKC(cudaMallocHost(&I->h_out, sizeof(double)));
+  CKC(cudaMalloc(&I->d_flag, sizeof(unsigned)));
   {
     std::vector<double> ones(I->p_pad, 1.0), r((size_t)category_count * eigen_count, 1.0),
         w((size_t)category_count * eigen_count, 1.0 / category_count),
@@ -436,6 +438,7 @@ int rrl_set_tip_states(int inst, int tip, const int32_t *states) {
   CK(cudaMemcpyAsync(I->d_states + (size_t)tip * I->p_pad, h.data(), I->p, cudaMemcpyHostToDevice,
                      I->stream));
   CK(cudaStreamSynchronize(I->stream));
+  if (!I->has_states[tip]) I->ops_valid = false;  // resolved descriptors name it as partials
   I->has_states[tip] = 1;
   return RRL_SUCCESS;
 }
@@ -445,12 +448,26 @@ int rrl_set_tip_states_u8(int inst, int first_tip, int count, const uint8_t *sta
   if (first_tip < 0 || count < 0 || first_tip + count > I->n_tips)
     return fail(RRL_ERROR_OUT_OF_RANGE, "tip range");
   if (!states) return fail(RRL_ERROR_GENERAL, "states NULL");
-  for (size_t i = 0; i < (size_t)count * I->p; ++i)
-    if (states[i] > I->s) return fail(RRL_ERROR_OUT_OF_RANGE, "state code > state_count");
-  CK(cudaMemcpy2DAsync(I->d_states + (size_t)first_tip * I->p_pad, I->p_pad, states, I->p, I->p,
-                       count, cudaMemcpyHostToDevice, I->stream));
+  if (count == 0) return RRL_SUCCESS;
+  // the rows go straight to the device (one DMA from a pinned caller buffer);
+  // the code range (<= s, s = missing) is checked there, not byte by byte on the host
+  uint8_t *dst = I->d_states + (size_t)first_tip * I->p_pad;
+  CK(cudaMemcpy2DAsync(dst, I->p_pad, states, I->p, I->p, count, cudaMemcpyHostToDevice, I->stream));
+  CK(static_cast<cudaError_t>(launch_check_states(dst, (size_t)count * I->p_pad, I->s, I->d_flag, I->stream)));
+  CK(cudaMemcpyAsync(I->h_out, I->d_flag, sizeof(unsigned), cudaMemcpyDeviceToHost, I->stream));
   CK(cudaStreamSynchronize(I->stream));
-  for (int t = first_tip; t < first_tip + count; ++t) I->has_states[t] = 1;
+  unsigned bad = 0;
+  std::memcpy(&bad, I->h_out, sizeof(unsigned));
+  for (int t = first_tip; t < first_tip + count; ++t) {
+    if (!I->has_states[t]) I->ops_valid = false;  // resolved descriptors name it as partials
+    I->has_states[t] = 1;
+  }
+  if (bad) {
+    // the rows are left as "missing" (all-ones) rather than holding out-of-range codes
+    CK(cudaMemset2DAsync(dst, I->p_pad, I->s, I->p, count, I->stream));
+    CK(cudaStreamSynchronize(I->stream));
+    return fail(RRL_ERROR_OUT_OF_RANGE, "state code > state_count");
+  }
   return RRL_SUCCESS;
 }
 

@@ -328,4 +328,28 @@ int launch_split_tf32(const float *x, float *lo, size_t n, void *stream) {
   return (int)cudaGetLastError();
 }
 
+// Tip-state validation on the device (rrl_set_tip_states_u8): any code > s in
+// `bytes` bytes (a multiple of 16: whole p_pad rows) sets *flag.  The padding
+// columns hold s (missing), which passes.
+__global__ void k_check_states(const uint4 *__restrict__ d, size_t n16, unsigned s, unsigned *__restrict__ flag) {
+  unsigned bad = 0;
+  const unsigned lim = s * 0x01010101u;
+  for (size_t i = blockIdx.x * (size_t)blockDim.x + threadIdx.x; i < n16; i += (size_t)gridDim.x * blockDim.x) {
+    const uint4 v = __ldg(d + i);
+    // per-byte unsigned compare: __vcmpgtu4 gives 0xff in every byte where v > s
+    bad |= __vcmpgtu4(v.x, lim) | __vcmpgtu4(v.y, lim) | __vcmpgtu4(v.z, lim) | __vcmpgtu4(v.w, lim);
+  }
+  if (__any_sync(0xffffffffu, bad != 0) && (threadIdx.x & 31) == 0) atomicOr(flag, 1u);
+}
+
+int launch_check_states(const uint8_t *d, size_t bytes, int s, unsigned *flag, void *stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  cudaError_t e = cudaMemsetAsync(flag, 0, sizeof(unsigned), st);
+  if (e != cudaSuccess || bytes == 0) return (int)e;
+  const size_t n16 = bytes / 16, blocks = (n16 + 255) / 256;
+  k_check_states<<<(unsigned)(blocks < 2368 ? blocks : 2368), 256, 0, st>>>(reinterpret_cast<const uint4 *>(d),
+                                                                           n16, (unsigned)s, flag);
+  return (int)cudaGetLastError();
+}
+
 }  // namespace rrl

@@ -56,6 +56,8 @@ int launch_split_tf32(const float *x, float *lo, size_t n, void *stream);
 int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
                                      int p_pad, const void *tmap_partials, const void *tmap_P,
                                      const void *tmap_Plo, void *stream);
+// *flag = 1 if any of `bytes` (multiple of 16) uint8 tip codes exceeds s, else 0.
+int launch_check_states(const uint8_t *d, size_t bytes, int s, unsigned *flag, void *stream);
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
                                int count, void *d_P, void *d_Plo, void *stream);

@@ -248,6 +248,29 @@ def test_tip_partials_equal_tip_states():
     tl.close()
 
 
+def test_tip_states_u8_validation_and_switch_back():
+    """Device-side code check of rrl_set_tip_states_u8 (code > s fails with
+    OUT_OF_RANGE, tips left all-missing); switching tips from partials back to
+    states re-resolves the cached descriptors."""
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="random", n=20, p=300, model="gtr", c=4, seed=10, missing_frac=0.1)
+    tl = gpu_setup(w, "reroot", 64)
+    a = tl.loglik()
+    for tip in (0, 3):
+        R.rrl_set_tip_partials(tl.inst, tip, pruning.tip_partials(w.tips[tip], 4))
+    tl.set_tips(w.tips)                       # back to states for every tip
+    assert rel(tl.loglik(), a) <= 1e-13
+    bad = w.tips.copy()
+    bad[5, 299] = 5                           # > s = 4
+    with pytest.raises(R.RRLError) as ei:
+        tl.set_tips(bad)
+    assert ei.value.code == R.ERROR_OUT_OF_RANGE
+    assert abs(tl.loglik()) <= 1e-9           # every tip left all-missing: lnL = 0
+    tl.set_tips(w.tips)
+    assert rel(tl.loglik(), a) <= 1e-13
+    tl.close()
+
+
 def test_pattern_weights():
     w = make_workload(tree_kind="random", n=25, p=400, model="gtr", c=4, seed=11)
     w.pattern_weights = np.random.default_rng(0).integers(1, 5, 400).astype(np.float64)
