@@ -316,7 +316,8 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
   I->mat_elems = (size_t)I->c * I->s_pad * I->s_pad;
   I->tip_partials.assign(tip_count, nullptr);
   I->has_states.assign(tip_count, 0);
-  I->nblocks = std::min(148 * 4, (pattern_count + 255) / 256);
+  // K4/K6 grid: a thread per pattern (4 states) or a warp per pattern (61 states)
+  I->nblocks = std::min(148 * 4, (pattern_count + (state_count == 61 ? 7 : 255)) / (state_count == 61 ? 8 : 256));
   auto bail = [&](int code, const std::string &m) {
     destroy(I);
     return fail(code, m);
@@ -939,7 +940,8 @@ static int root_common(Instance *I, int root_buffer, int cat_weights_idx, int fr
   const int32_t *cum = cumulative_idx >= 0 ? I->d_scale + (size_t)cumulative_idx * I->p_pad + pb : nullptr;
   const size_t pel = (I->s == 4 ? (size_t)I->c * 4 : (size_t)I->s_pad) * pb * I->elt;
   const int np = pe - pb;
-  const int nb = std::max(1, std::min(I->nblocks, (np + 255) / 256));
+  const int per_block = I->s == 61 ? 8 : 256;  // patterns per K4 block (a warp per codon pattern)
+  const int nb = std::max(1, std::min(I->nblocks, (np + per_block - 1) / per_block));
   {
     Timed tm(I, 2);
     CKL(launch_root_lnl(I->prec, I->s, I->s_pad, I->c, static_cast<const char *>(root) + pel,

@@ -58,38 +58,40 @@ __device__ inline float tf32_lo(float x) {  // rn_tf32(x - trunc_tf32(x)), the 3
 
 template <typename T>
 __global__ void __launch_bounds__(256)
-k_transition64(int s, int C, const double *__restrict__ eig, const double *__restrict__ rates,
+k_transition64(int s, int C, int items, const double *__restrict__ eig, const double *__restrict__ rates,
                const int32_t *__restrict__ idx, const double *__restrict__ tlen, T *__restrict__ P,
                float *__restrict__ Plo) {
+  // Persistent: V and V^-1 (the same for every matrix) are staged in shared
+  // memory once per block, which then walks (matrix, category) items.
   extern __shared__ double sm[];
   double *Vt = sm;              // [64 k][64 z]
   double *Vi = sm + 64 * 64;    // [64 k][64 x]
-  double *ex = sm + 2 * 64 * 64;  // [C][64]
-  const int m = blockIdx.x, c = blockIdx.y, tid = threadIdx.x;
+  double *ex = sm + 2 * 64 * 64;  // [64]
+  const int tid = threadIdx.x;
   const double *lam = eig + 2 * s * s;
   for (int i = tid; i < 64 * 64; i += 256) {
-    const int a = i >> 6, b = i & 63;  // a = row, b = column of the padded matrix
-    Vt[b * 64 + a] = (a < s && b < s) ? eig[a * s + b] : 0.0;        // V[a][b] -> Vt[k=b][z=a]
-    Vi[i] = (a < s && b < s) ? eig[s * s + a * s + b] : 0.0;         // Vinv[k=a][x=b]
+    const int k = i >> 6, q = i & 63;  // consecutive threads: consecutive shared-memory words
+    Vt[i] = (k < s && q < s) ? eig[q * s + k] : 0.0;          // V[z=q][k] -> Vt[k][z]
+    Vi[i] = (k < s && q < s) ? eig[s * s + k * s + q] : 0.0;  // Vinv[k][x=q]
   }
-  const double rt = rates[c] * tlen[m];
-  for (int k = tid; k < 64; k += 256) ex[k] = k < s ? exp(lam[k] * rt) : 0.0;
-  __syncthreads();
   const int z0 = (tid >> 4) * 4, x0 = (tid & 15) * 4;
-  {
+  for (int it = blockIdx.x; it < items; it += gridDim.x) {
+    const int m = it / C, c = it - m * C;
+    __syncthreads();  // V staged / the previous item's ex consumed
+    if (tid < 64) ex[tid] = tid < s ? exp(lam[tid] * (rates[c] * tlen[m])) : 0.0;
+    __syncthreads();
     double acc[4][4];
 #pragma unroll
     for (int i = 0; i < 4; ++i)
 #pragma unroll
       for (int j = 0; j < 4; ++j) acc[i][j] = 0.0;
-    const double *e = ex;
 #pragma unroll 4
     for (int k = 0; k < s; ++k) {
       const double2 va = *reinterpret_cast<const double2 *>(Vt + k * 64 + z0);
       const double2 vb = *reinterpret_cast<const double2 *>(Vt + k * 64 + z0 + 2);
       const double2 wa = *reinterpret_cast<const double2 *>(Vi + k * 64 + x0);
       const double2 wb = *reinterpret_cast<const double2 *>(Vi + k * 64 + x0 + 2);
-      const double ek = e[k];
+      const double ek = ex[k];
       const double a[4] = {va.x * ek, va.y * ek, vb.x * ek, vb.y * ek};
       const double b[4] = {wa.x, wa.y, wb.x, wb.y};
 #pragma unroll
@@ -99,13 +101,19 @@ k_transition64(int s, int C, const double *__restrict__ eig, const double *__res
     }
     const size_t off = ((size_t)idx[m] * C + c) * 64 * 64;
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
-#pragma unroll
-      for (int j = 0; j < 4; ++j) {
-        const T v = (T)acc[i][j];
-        P[off + (z0 + i) * 64 + x0 + j] = v;
-        if (Plo != nullptr) Plo[off + (z0 + i) * 64 + x0 + j] = tf32_lo((float)v);
+    for (int i = 0; i < 4; ++i) {
+      T *row = P + off + (z0 + i) * 64 + x0;
+      if constexpr (sizeof(T) == 4) {
+        const float4 v = make_float4((float)acc[i][0], (float)acc[i][1], (float)acc[i][2], (float)acc[i][3]);
+        *reinterpret_cast<float4 *>(row) = v;
+        if (Plo != nullptr)
+          *reinterpret_cast<float4 *>(Plo + off + (z0 + i) * 64 + x0) =
+              make_float4(tf32_lo(v.x), tf32_lo(v.y), tf32_lo(v.z), tf32_lo(v.w));
+      } else {
+        reinterpret_cast<double2 *>(row)[0] = make_double2(acc[i][0], acc[i][1]);
+        reinterpret_cast<double2 *>(row)[1] = make_double2(acc[i][2], acc[i][3]);
       }
+    }
   }
 }
 
@@ -187,6 +195,31 @@ k_root(const T *__restrict__ L, int s, int s_pad, int C, const double *__restric
        double *__restrict__ blocks, unsigned *__restrict__ count, double *__restrict__ out) {
   __shared__ double red[32];
   double part = 0.0;
+  if (s_pad == 64) {
+    // 61 states ([c][p_pad][64] rows of 256 B): one warp per pattern, lanes over
+    // states (coalesced row reads), a fixed-order shuffle reduction
+    const int lane = threadIdx.x & 31;
+    const int nw = (gridDim.x * blockDim.x) >> 5;
+    for (int i = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; i < p; i += nw) {
+      double a = 0.0;
+      for (int c = 0; c < C; ++c) {
+        const T *row = L + ((size_t)c * p_pad + i) * 64;
+        double sc = lane < s ? pi[lane] * (double)row[lane] : 0.0;
+        if (lane + 32 < s) sc = fma(pi[lane + 32], (double)row[lane + 32], sc);
+        a = fma(w[c], sc, a);
+      }
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(0xffffffffu, a, o);
+      if (lane == 0) {
+        double l = log(a);
+        if (cum != nullptr) l += (double)cum[i] * kLn2;
+        site[i] = l;
+        part += pw[i] * l;
+      }
+    }
+    finish_sum(part, red, blocks, count, out);
+    return;
+  }
   for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < p; i += gridDim.x * blockDim.x) {
     const double a = site_root(L, s, s_pad, C, i, p_pad, w, pi);
     double l = log(a);
@@ -248,18 +281,26 @@ int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *
                                int count, void *d_P, void *d_Plo, void *stream) {
   if (count <= 0) return 0;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (s_pad == 64) {  // codon: register-tiled, one block per matrix
+  if (s_pad == 64) {  // codon: register-tiled, persistent blocks over (matrix, category) items
     const size_t smem64 = sizeof(double) * (2 * 64 * 64 + 64);
-    if (prec == 32) {
+    const int items = count * c;
+    static int grid_cap = 0;
+    if (grid_cap == 0) {
+      int dev = 0, nsm = 0, per = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
       cudaFuncSetAttribute(k_transition64<float>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
-      k_transition64<float><<<dim3(count, c), 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx, d_t,
-                                                                 static_cast<float *>(d_P),
-                                                                 static_cast<float *>(d_Plo));
-    } else {
       cudaFuncSetAttribute(k_transition64<double>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem64);
-      k_transition64<double><<<dim3(count, c), 256, smem64, st>>>(s, c, d_eig, d_rates, d_idx, d_t,
-                                                                  static_cast<double *>(d_P), nullptr);
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_transition64<double>, 256, smem64);
+      grid_cap = nsm * (per > 0 ? per : 1);
     }
+    const int grid = items < grid_cap ? items : grid_cap;
+    if (prec == 32)
+      k_transition64<float><<<grid, 256, smem64, st>>>(s, c, items, d_eig, d_rates, d_idx, d_t,
+                                                       static_cast<float *>(d_P), static_cast<float *>(d_Plo));
+    else
+      k_transition64<double><<<grid, 256, smem64, st>>>(s, c, items, d_eig, d_rates, d_idx, d_t,
+                                                        static_cast<double *>(d_P), nullptr);
     return (int)cudaGetLastError();
   }
   const size_t smem = sizeof(double) * (2 * s * s + s);
