@@ -12,15 +12,15 @@
 // One CTA = one (operation, 64-pattern tile) for ALL categories, because the
 // per-pattern rescale (reading A5) takes the max over
 // (c, z).  256 threads: thread (pg, zg) owns patterns 4pg..4pg+3 and states
-// 4zg..4zg+3, a 4x4 register tile per child; per k step it reads 4+4 child
-// values (padded rows, conflict-free) and two 128-bit rows of P^T from
-// shared memory for 32 FMAs.  The category results stay in registers until
-// the cross-category max is known (16-lane shuffle), then are scaled by the
-// exact power of two and stored.
+// 4zg..4zg+3, a 4x4 register tile; one child at a time sits in shared memory
+// (per k step: 4 child values, padded rows, conflict-free, and a row of P^T
+// for 16 FMAs).  Each category's unscaled product is stored at once and a
+// running max over (c, z) kept; when the max is known (16-lane shuffle) the
+// thread scales the values it stored by the exact power of two.
 //
-// This is the FP32/FP64 SIMT path (ALU-bound: ~15 k flop per pattern-op at
-// c = 4).  The tcgen05 tensor-core variant of the same contraction is the
-// next step.
+// This is the FP64 (and RRL_FLAG_CODON_SIMT fp32) path, ALU-bound: ~15 k
+// flop per pattern-op at c = 4.  fp32 runs on the tcgen05 kernels
+// (kernels_codon_tc5.cu, kernels_codon_tc.cu).
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -65,13 +65,51 @@ __device__ inline double pow2_neg(double, int e) {
 
 template <typename T>
 struct CodonSmem {
-  T A[2][kTP * kAStride];     // child tiles, pattern-major, padded rows
-  T Pt[2][kPRows * kPS];      // P^T per child: Pt[x][z] = P[z][x]; row 64 = row sums
-  uint8_t st[2][kTP];         // tip states
+  T A[kTP * kAStride];   // one child tile, pattern-major, padded rows
+  T Pt[kPRows * kPS];    // that child's P^T: Pt[x][z] = P[z][x]; row 64 = row sums
+  uint8_t st[2][kTP];    // tip states
 };
 
+// One child (b) of category c for this thread's 4x4 (pattern, state) tile.
+template <typename T>
+__device__ inline void codon_child(CodonSmem<T> &sm, bool tip, int b, int pg, int zg, T (&acc)[4][4]) {
+  if (tip) {
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const unsigned s = sm.st[b][pg * 4 + i];
+      const int row = s < (unsigned)kS ? (int)s : 64;
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc[i][j] = sm.Pt[row * kPS + zg * 4 + j];
+    }
+    return;
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i)
+#pragma unroll
+    for (int j = 0; j < 4; ++j) acc[i][j] = T(0);
+  const T *Ab = &sm.A[(pg * 4) * kAStride];
+  const T *Pb = &sm.Pt[zg * 4];
+#pragma unroll 4
+  for (int x = 0; x < kS; ++x) {
+    T a[4], w[4];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) a[i] = Ab[i * kAStride + x];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) w[j] = Pb[x * kPS + j];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+      for (int j = 0; j < 4; ++j) acc[i][j] = fma(a[i], w[j], acc[i][j]);
+  }
+}
+
+// One child at a time in shared memory (68 KB in fp64, so two or three CTAs
+// share an SM); each category's unscaled product goes straight to the output
+// buffer while a running max over (c, z) is kept, and once the pattern's
+// exponent is known the thread re-reads (L1/L2) and scales the values it wrote
+// itself -- no per-category register file, no cross-thread hazard.
 template <typename T, int C>
-__global__ void __launch_bounds__(kThreads3)
+__global__ void __launch_bounds__(kThreads3, sizeof(T) == 8 ? 2 : 3)
 k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
   extern __shared__ __align__(16) unsigned char smem_raw3[];
   CodonSmem<T> &sm = *reinterpret_cast<CodonSmem<T> *>(smem_raw3);
@@ -94,98 +132,77 @@ k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
       sm.st[b][tid] = pp < p ? static_cast<const uint8_t *>(in[b])[pp] : (uint8_t)kS;
     }
 
-  T res[C][4][4];
+  // exponents known up front (stored factors) are applied in the first pass
+  const bool two_pass = op.scale_out != nullptr;
+  T f_in[4];
 #pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int pp = p0 + pg * 4 + i;
+    f_in[i] = (!two_pass && op.scale_in != nullptr && pp < p) ? pow2_neg(T(0), op.scale_in[pp]) : T(1);
+  }
+  T *out = static_cast<T *>(op.out);
+  T m[4] = {T(0), T(0), T(0), T(0)};
   for (int c = 0; c < C; ++c) {
-    __syncthreads();  // previous category's tiles are no longer read
-    // ---- stage P^T (both children) and the child tiles
+    T prod[4][4];
     for (int b = 0; b < 2; ++b) {
+      __syncthreads();  // the previous child's tiles are no longer read
       const T *P = Pg[b] + (size_t)c * kSP * kSP;
       for (int i = tid; i < kSP * kSP; i += kThreads3) {
         const int z = i / kSP, x = i % kSP;
-        sm.Pt[b][x * kPS + z] = P[i];
+        sm.Pt[x * kPS + z] = P[i];
       }
       if (!tip[b]) {
         const T *A = static_cast<const T *>(in[b]) + ((size_t)c * p_pad + p0) * kSP;
         for (int i = tid; i < kTP * kSP; i += kThreads3) {
           const int pp = i / kSP, x = i % kSP;
-          sm.A[b][pp * kAStride + x] = A[i];  // rows beyond p exist (p_pad) and are never stored
+          sm.A[pp * kAStride + x] = A[i];  // rows beyond p exist (p_pad) and are never stored
         }
       }
-    }
-    __syncthreads();
-    for (int b = 0; b < 2; ++b)  // row sums (tip code >= 61 = missing)
-      if (tip[b] && tid < kSP) {
-        T acc = T(0);
-        for (int x = 0; x < kSP; ++x) acc += sm.Pt[b][x * kPS + tid];
-        sm.Pt[b][64 * kPS + tid] = acc;
-      }
-    __syncthreads();
-    // ---- two 4x4 register tiles
-    T acc[2][4][4];
-#pragma unroll
-    for (int b = 0; b < 2; ++b) {
-      if (tip[b]) {
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const unsigned s = sm.st[b][pg * 4 + i];
-          const int row = s < (unsigned)kS ? (int)s : 64;
-#pragma unroll
-          for (int j = 0; j < 4; ++j) acc[b][i][j] = sm.Pt[b][row * kPS + zg * 4 + j];
+      __syncthreads();
+      if (tip[b]) {  // row sums (tip code >= 61 = missing)
+        if (tid < kSP) {
+          T acc = T(0);
+          for (int x = 0; x < kSP; ++x) acc += sm.Pt[x * kPS + tid];
+          sm.Pt[64 * kPS + tid] = acc;
         }
-      } else {
-#pragma unroll
-        for (int i = 0; i < 4; ++i)
-#pragma unroll
-          for (int j = 0; j < 4; ++j) acc[b][i][j] = T(0);
-        const T *Ab = &sm.A[b][(pg * 4) * kAStride];
-        const T *Pb = &sm.Pt[b][zg * 4];
-#pragma unroll 4
-        for (int x = 0; x < kS; ++x) {
-          T a[4], w[4];
-#pragma unroll
-          for (int i = 0; i < 4; ++i) a[i] = Ab[i * kAStride + x];
-#pragma unroll
-          for (int j = 0; j < 4; ++j) w[j] = Pb[x * kPS + j];
-#pragma unroll
-          for (int i = 0; i < 4; ++i)
-#pragma unroll
-            for (int j = 0; j < 4; ++j) acc[b][i][j] = fma(a[i], w[j], acc[b][i][j]);
-        }
+        __syncthreads();
       }
+      T acc[4][4];
+      codon_child(sm, tip[b], b, pg, zg, acc);
+#pragma unroll
+      for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) prod[i][j] = b == 0 ? acc[i][j] : prod[i][j] * acc[i][j];
     }
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < 4; ++i) {
+      const int pp = p0 + pg * 4 + i;
 #pragma unroll
-      for (int j = 0; j < 4; ++j) res[c][i][j] = acc[0][i][j] * acc[1][i][j];
+      for (int j = 0; j < 4; ++j) m[i] = fmax(m[i], prod[i][j]);
+      if (pp < p) {
+        T *dst = out + ((size_t)c * p_pad + pp) * kSP + zg * 4;
+#pragma unroll
+        for (int j = 0; j < 4; ++j) dst[j] = prod[i][j] * f_in[i];
+      }
+    }
   }
+  if (!two_pass) return;
 
-  // ---- rescale: max over (c, z) per pattern across the 16 zg lanes
-  T *out = static_cast<T *>(op.out);
+  // ---- rescale: max over (c, z) per pattern across the 16 zg lanes, then the
+  // thread scales the values it stored above by the exact power of two
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
     const int pp = p0 + pg * 4 + i;
     const bool valid = pp < p;
-    int e = 0;
-    if (op.scale_out != nullptr || op.scale_in != nullptr) {
-      if (op.scale_out != nullptr) {
-        T m = T(0);
+    T mm = m[i];
 #pragma unroll
-        for (int c = 0; c < C; ++c)
-#pragma unroll
-          for (int j = 0; j < 4; ++j) m = fmax(m, res[c][i][j]);
-#pragma unroll
-        for (int o = 1; o < 16; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
-        e = frexp_exp3(m);
-        if (valid && zg == 0) {
-          int tot = e;
-          if (op.cum1 != nullptr) tot += op.cum1[pp];
-          if (op.cum2 != nullptr) tot += op.cum2[pp];
-          op.scale_out[pp] = tot;
-        }
-      } else {
-        e = valid ? op.scale_in[pp] : 0;
-      }
+    for (int o = 1; o < 16; o <<= 1) mm = fmax(mm, __shfl_xor_sync(0xffffffffu, mm, o));
+    const int e = frexp_exp3(mm);
+    if (valid && zg == 0) {
+      int tot = e;
+      if (op.cum1 != nullptr) tot += op.cum1[pp];
+      if (op.cum2 != nullptr) tot += op.cum2[pp];
+      op.scale_out[pp] = tot;
     }
     const T f = pow2_neg(T(0), e);
     if (valid) {
@@ -193,7 +210,7 @@ k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
       for (int c = 0; c < C; ++c) {
         T *dst = out + ((size_t)c * p_pad + pp) * kSP + zg * 4;
 #pragma unroll
-        for (int j = 0; j < 4; ++j) dst[j] = res[c][i][j] * f;
+        for (int j = 0; j < 4; ++j) dst[j] = dst[j] * f;
       }
     }
   }
