@@ -12,7 +12,7 @@
 // One CTA = one (operation, 64-pattern tile) for ALL categories, because the
 // per-pattern rescale (reading A5) takes the max over
 // (c, z).  256 threads: thread (pg, zg) owns patterns 4pg..4pg+3 and states
-// 4zg..4zg+3, a 4x4 register tile; one child at a time sits in shared memory
+// {2zg, 2zg+1, 32+2zg, 33+2zg}, a 4x4 register tile; one child at a time sits in shared memory
 // (per k step: 4 child values, padded rows, conflict-free, and a row of P^T
 // for 16 FMAs).  Each category's unscaled product is stored at once and a
 // running max over (c, z) kept; when the max is known (16-lane shuffle) the
@@ -70,6 +70,25 @@ struct CodonSmem {
   uint8_t st[2][kTP];    // tip states
 };
 
+// State j (0..3) of thread group zg: {2zg, 2zg+1, 32+2zg, 33+2zg}, so that the
+// 16 groups' pairs are contiguous (conflict-free 2-element shared loads,
+// coalesced stores).
+__device__ inline int zcol(int zg, int j) { return (j < 2 ? 0 : 32) + 2 * zg + (j & 1); }
+
+template <typename T> struct Pair;
+template <> struct Pair<float> {
+  __device__ static inline void ld(const float *p, float &a, float &b) {
+    const float2 v = *reinterpret_cast<const float2 *>(p);
+    a = v.x; b = v.y;
+  }
+};
+template <> struct Pair<double> {
+  __device__ static inline void ld(const double *p, double &a, double &b) {
+    const double2 v = *reinterpret_cast<const double2 *>(p);
+    a = v.x; b = v.y;
+  }
+};
+
 // One child (b) of category c for this thread's 4x4 (pattern, state) tile.
 template <typename T>
 __device__ inline void codon_child(CodonSmem<T> &sm, bool tip, int b, int pg, int zg, T (&acc)[4][4]) {
@@ -78,8 +97,8 @@ __device__ inline void codon_child(CodonSmem<T> &sm, bool tip, int b, int pg, in
     for (int i = 0; i < 4; ++i) {
       const unsigned s = sm.st[b][pg * 4 + i];
       const int row = s < (unsigned)kS ? (int)s : 64;
-#pragma unroll
-      for (int j = 0; j < 4; ++j) acc[i][j] = sm.Pt[row * kPS + zg * 4 + j];
+      Pair<T>::ld(&sm.Pt[row * kPS + 2 * zg], acc[i][0], acc[i][1]);
+      Pair<T>::ld(&sm.Pt[row * kPS + 32 + 2 * zg], acc[i][2], acc[i][3]);
     }
     return;
   }
@@ -88,14 +107,14 @@ __device__ inline void codon_child(CodonSmem<T> &sm, bool tip, int b, int pg, in
 #pragma unroll
     for (int j = 0; j < 4; ++j) acc[i][j] = T(0);
   const T *Ab = &sm.A[(pg * 4) * kAStride];
-  const T *Pb = &sm.Pt[zg * 4];
+  const T *Pb = &sm.Pt[2 * zg];
 #pragma unroll 4
   for (int x = 0; x < kS; ++x) {
     T a[4], w[4];
 #pragma unroll
     for (int i = 0; i < 4; ++i) a[i] = Ab[i * kAStride + x];
-#pragma unroll
-    for (int j = 0; j < 4; ++j) w[j] = Pb[x * kPS + j];
+    Pair<T>::ld(Pb + x * kPS, w[0], w[1]);
+    Pair<T>::ld(Pb + x * kPS + 32, w[2], w[3]);
 #pragma unroll
     for (int i = 0; i < 4; ++i)
 #pragma unroll
@@ -147,9 +166,9 @@ k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
     for (int b = 0; b < 2; ++b) {
       __syncthreads();  // the previous child's tiles are no longer read
       const T *P = Pg[b] + (size_t)c * kSP * kSP;
-      for (int i = tid; i < kSP * kSP; i += kThreads3) {
-        const int z = i / kSP, x = i % kSP;
-        sm.Pt[x * kPS + z] = P[i];
+      for (int i = tid; i < kSP * kSP; i += kThreads3) {  // consecutive threads: consecutive z (conflict-free)
+        const int z = i % kSP, x = i / kSP;
+        sm.Pt[x * kPS + z] = __ldg(P + z * kSP + x);
       }
       if (!tip[b]) {
         const T *A = static_cast<const T *>(in[b]) + ((size_t)c * p_pad + p0) * kSP;
@@ -180,9 +199,9 @@ k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
 #pragma unroll
       for (int j = 0; j < 4; ++j) m[i] = fmax(m[i], prod[i][j]);
       if (pp < p) {
-        T *dst = out + ((size_t)c * p_pad + pp) * kSP + zg * 4;
+        T *dst = out + ((size_t)c * p_pad + pp) * kSP;
 #pragma unroll
-        for (int j = 0; j < 4; ++j) dst[j] = prod[i][j] * f_in[i];
+        for (int j = 0; j < 4; ++j) dst[zcol(zg, j)] = prod[i][j] * f_in[i];
       }
     }
   }
@@ -208,9 +227,9 @@ k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
     if (valid) {
 #pragma unroll
       for (int c = 0; c < C; ++c) {
-        T *dst = out + ((size_t)c * p_pad + pp) * kSP + zg * 4;
+        T *dst = out + ((size_t)c * p_pad + pp) * kSP;
 #pragma unroll
-        for (int j = 0; j < 4; ++j) dst[j] = dst[j] * f;
+        for (int j = 0; j < 4; ++j) dst[zcol(zg, j)] = dst[zcol(zg, j)] * f;
       }
     }
   }

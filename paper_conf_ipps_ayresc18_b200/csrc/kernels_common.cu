@@ -74,7 +74,9 @@ k_transition64(int s, int C, int items, const double *__restrict__ eig, const do
     Vt[i] = (k < s && q < s) ? eig[q * s + k] : 0.0;          // V[z=q][k] -> Vt[k][z]
     Vi[i] = (k < s && q < s) ? eig[s * s + k * s + q] : 0.0;  // Vinv[k][x=q]
   }
-  const int z0 = (tid >> 4) * 4, x0 = (tid & 15) * 4;
+  // thread: rows z0..z0+3, columns {2l, 2l+1, 32+2l, 33+2l} (l = tid & 15), so a
+  // half-warp's column pairs are contiguous (conflict-free double2 loads)
+  const int z0 = (tid >> 4) * 4, x0 = (tid & 15) * 2;
   for (int it = blockIdx.x; it < items; it += gridDim.x) {
     const int m = it / C, c = it - m * C;
     __syncthreads();  // V staged / the previous item's ex consumed
@@ -90,7 +92,7 @@ k_transition64(int s, int C, int items, const double *__restrict__ eig, const do
       const double2 va = *reinterpret_cast<const double2 *>(Vt + k * 64 + z0);
       const double2 vb = *reinterpret_cast<const double2 *>(Vt + k * 64 + z0 + 2);
       const double2 wa = *reinterpret_cast<const double2 *>(Vi + k * 64 + x0);
-      const double2 wb = *reinterpret_cast<const double2 *>(Vi + k * 64 + x0 + 2);
+      const double2 wb = *reinterpret_cast<const double2 *>(Vi + k * 64 + 32 + x0);
       const double ek = ex[k];
       const double a[4] = {va.x * ek, va.y * ek, vb.x * ek, vb.y * ek};
       const double b[4] = {wa.x, wa.y, wb.x, wb.y};
@@ -104,14 +106,18 @@ k_transition64(int s, int C, int items, const double *__restrict__ eig, const do
     for (int i = 0; i < 4; ++i) {
       T *row = P + off + (z0 + i) * 64 + x0;
       if constexpr (sizeof(T) == 4) {
-        const float4 v = make_float4((float)acc[i][0], (float)acc[i][1], (float)acc[i][2], (float)acc[i][3]);
-        *reinterpret_cast<float4 *>(row) = v;
-        if (Plo != nullptr)
-          *reinterpret_cast<float4 *>(Plo + off + (z0 + i) * 64 + x0) =
-              make_float4(tf32_lo(v.x), tf32_lo(v.y), tf32_lo(v.z), tf32_lo(v.w));
+        const float2 va = make_float2((float)acc[i][0], (float)acc[i][1]);
+        const float2 vb = make_float2((float)acc[i][2], (float)acc[i][3]);
+        *reinterpret_cast<float2 *>(row) = va;
+        *reinterpret_cast<float2 *>(row + 32) = vb;
+        if (Plo != nullptr) {
+          float *lo = Plo + off + (z0 + i) * 64 + x0;
+          *reinterpret_cast<float2 *>(lo) = make_float2(tf32_lo(va.x), tf32_lo(va.y));
+          *reinterpret_cast<float2 *>(lo + 32) = make_float2(tf32_lo(vb.x), tf32_lo(vb.y));
+        }
       } else {
-        reinterpret_cast<double2 *>(row)[0] = make_double2(acc[i][0], acc[i][1]);
-        reinterpret_cast<double2 *>(row)[1] = make_double2(acc[i][2], acc[i][3]);
+        *reinterpret_cast<double2 *>(row) = make_double2(acc[i][0], acc[i][1]);
+        *reinterpret_cast<double2 *>(row + 32) = make_double2(acc[i][2], acc[i][3]);
       }
     }
   }
