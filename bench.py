@@ -68,13 +68,31 @@ def bytes_per_pass(ops, n, p, c, s, elt, cumulative=True):
 
 # ----------------------------------------------------------------------------- clocks
 class ClockSampler:
+    """SM clocks and throttle reasons during the timed region: NVML polled every
+    5 ms from a thread (plus `sample()` calls the timing loop makes while the
+    GPU is still busy with enqueued steps, so even a short region is covered);
+    nvidia-smi -lms 100 when NVML is unavailable."""
     FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
     def __init__(self, device: int):
-        self.rows = []
-        self.proc = None
+        self.rows, self.proc, self.nv, self.t = [], None, None, None
+        self._stop = threading.Event()
+        try:
+            import pynvml as nv
+            nv.nvmlInit()
+            self.h = nv.nvmlDeviceGetHandleByIndex(device)
+            self.nv = nv
+            self.bits = [nv.nvmlClocksEventReasonHwSlowdown, nv.nvmlClocksEventReasonHwThermalSlowdown,
+                         nv.nvmlClocksEventReasonSwThermalSlowdown, nv.nvmlClocksEventReasonSwPowerCap]
+            self.max_mhz = float(nv.nvmlDeviceGetMaxClockInfo(self.h, nv.NVML_CLOCK_SM))
+            self.t = threading.Thread(target=self._poll, daemon=True)
+            self.t.start()
+            return
+        except Exception:
+            self.nv = None
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
@@ -85,36 +103,49 @@ class ClockSampler:
         except Exception:
             self.proc = None
 
+    def sample(self):
+        if self.nv is None:
+            return
+        try:
+            sm = float(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+            r = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+            self.rows.append((sm, self.max_mhz, [bool(r & b) for b in self.bits]))
+        except Exception:
+            pass
+
+    def _poll(self):
+        while not self._stop.wait(0.005):
+            self.sample()
+
     def _read(self):
         for line in self.proc.stdout:
-            self.rows.append(line.strip())
-
-    def stop(self) -> dict:
-        if self.proc is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=5)
-        except Exception:
-            self.proc.kill()
-        self.t.join(timeout=2)
-        sm, mx, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for r in self.rows:
-            parts = [x.strip() for x in r.split(",")]
+            parts = [x.strip() for x in line.strip().split(",")]
             if len(parts) != 6:
                 continue
             try:
-                sm.append(float(parts[0]))
-                mx.append(float(parts[1]))
+                self.rows.append((float(parts[0]), float(parts[1]), [v.lower() == "active" for v in parts[2:]]))
             except ValueError:
                 continue
-            for nm, v in zip(names, parts[2:]):
-                if v.lower() == "active":
-                    reasons.add(nm)
+
+    def stop(self) -> dict:
+        if self.nv is None and self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self._stop.set()
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+        if self.t is not None:
+            self.t.join(timeout=2)
+        rows = list(self.rows)
+        sm = [r[0] for r in rows]
+        reasons = sorted({nm for r in rows for nm, on in zip(self.NAMES, r[2]) if on})
         return {"sm_mhz": float(np.median(sm)) if sm else None,
-                "sm_max_mhz": float(max(mx)) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+                "sm_max_mhz": float(max(r[1] for r in rows)) if rows else None,
+                "reasons": reasons, "samples": len(sm),
+                "source": "nvml" if self.nv is not None else "nvidia-smi"}
 
 
 # ----------------------------------------------------------------------------- helpers
@@ -309,7 +340,7 @@ def main():
         if dist is not None:
             allreduce_(d_out)
 
-    def timed(tl, steps, warmup):
+    def timed(tl, steps, warmup, clocks=None):
         """Per-step CUDA events on the launching stream; L2 flushed before
         every step outside the events; barrier + synchronize on both sides."""
         for _ in range(warmup):
@@ -325,11 +356,15 @@ def main():
         # replay of the updatePartials region (the roofline's launch durations)
         R.rrl_set_profiling(tl.inst, True)
         R.rrl_reset_profile(tl.inst)
-        for a, b in evs:
+        for i, (a, b) in enumerate(evs):
             flush.zero_()
             a.record(stream)
             step(tl)
             b.record(stream)
+            if clocks is not None and i % 16 == 15:
+                clocks.sample()  # the GPU is still running enqueued steps
+        if clocks is not None:
+            clocks.sample()
         torch.cuda.synchronize()
         if dist is not None:
             dist.barrier()
@@ -347,7 +382,7 @@ def main():
         tl = make(w, "reroot", precision, reuse)
         sched = tl.sched
         clocks = ClockSampler(local)
-        ms, prof = timed(tl, steps, warmup)
+        ms, prof = timed(tl, steps, warmup, clocks)
         launches = prof["kernel_launches"]
         clk = clocks.stop()
         fl = flops_per_pass(n, p, c, s)

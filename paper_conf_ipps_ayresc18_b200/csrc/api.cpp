@@ -67,8 +67,9 @@ struct Instance {
   int nblocks = 0;
 
   // transition-matrix call staging
+  double *d_t = nullptr;       // [t_cap] branch lengths, then d_midx [t_cap] (one allocation)
   int32_t *d_midx = nullptr;
-  double *d_t = nullptr;
+  std::vector<char> h_tstage;  // host staging of the same layout: one H2D copy per call
   int t_cap = 0;
   // accumulate-scale index list
   int32_t *d_sidx = nullptr;
@@ -198,7 +199,7 @@ void destroy(Instance *I) {
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
                   I->d_catw,     I->d_freqs,  I->d_pw,   I->d_site,  I->d_block, I->d_out, I->d_count,
-                  I->d_midx,     I->d_t,      I->d_sidx, I->d_ops,  I->d_Plo,  I->d_flag};
+                  I->d_t,      I->d_sidx, I->d_ops,  I->d_Plo,  I->d_flag};
   for (void *q : ptrs)
     if (q) cudaFree(q);
   if (I->h_ops) cudaFreeHost(I->h_ops);
@@ -593,18 +594,23 @@ int rrl_update_transition_matrices(int inst, int eigen_idx, const int32_t *matri
     if (matrix_idx[i] < 0 || matrix_idx[i] >= I->n_mat) return fail(RRL_ERROR_OUT_OF_RANGE, "matrix index");
   if (count > I->t_cap) {
     CK(cudaStreamSynchronize(I->stream));
-    if (I->d_midx) cudaFree(I->d_midx);
     if (I->d_t) cudaFree(I->d_t);
-    I->d_midx = nullptr;
     I->d_t = nullptr;
-    CK(cudaMalloc(&I->d_midx, sizeof(int32_t) * count));
-    CK(cudaMalloc(&I->d_t, sizeof(double) * count));
+    I->d_midx = nullptr;
+    const size_t bytes = (sizeof(double) + sizeof(int32_t)) * (size_t)count;
+    CK(cudaMalloc(&I->d_t, bytes));
+    I->h_tstage.resize(bytes);
+    I->d_midx = reinterpret_cast<int32_t *>(I->d_t + count);
     I->t_cap = count;
   }
-  // cudaMemcpyAsync from pageable memory is staged synchronously by the driver,
-  // so the caller's arrays may be released on return.
-  CK(cudaMemcpyAsync(I->d_midx, matrix_idx, sizeof(int32_t) * count, cudaMemcpyHostToDevice, I->stream));
-  CK(cudaMemcpyAsync(I->d_t, t, sizeof(double) * count, cudaMemcpyHostToDevice, I->stream));
+  // [t | matrix_idx] packed, one H2D copy.  A copy from pageable memory is
+  // staged by the driver before cudaMemcpyAsync returns, so neither the
+  // caller's arrays nor h_tstage are referenced after return.
+  double *ht = reinterpret_cast<double *>(I->h_tstage.data());
+  std::memcpy(ht, t, sizeof(double) * count);
+  std::memcpy(ht + I->t_cap, matrix_idx, sizeof(int32_t) * count);
+  CK(cudaMemcpyAsync(I->d_t, ht, (sizeof(double) + sizeof(int32_t)) * (size_t)I->t_cap, cudaMemcpyHostToDevice,
+                     I->stream));
   const size_t eig_sz = 2 * (size_t)I->s * I->s + I->s;
   {
     Timed tm(I, 1);
