@@ -403,6 +403,38 @@ __device__ inline void load_ptables_consumers(T (*sP)[C][kPTab], const DevOp &op
   consumer_sync();
 }
 
+// Both children tips: a pattern's whole output (every category, scaled) and its
+// exponent depend only on the pair of state codes, so the consumers evaluate
+// the 5 x 5 pairs once per operation with exactly the per-item arithmetic
+// (column lookups, product, max over (c, z), exact 2^-e) and each item becomes
+// a table read.  tab: [25][C][4], tabe: [25].
+template <typename T, int C, int SCALE>
+__device__ inline void build_tiptip_table(T (*sP)[C][kPTab], T *tab, int *tabe) {
+  const int t = threadIdx.x;
+  if (t < ((25 * C + 31) / 32) * 32) {  // whole warps (the max is a C-lane shuffle)
+    const int cat = t % C, combo = min(t / C, 24);
+    const unsigned s1 = (unsigned)(combo / 5), s2 = (unsigned)(combo % 5);
+    T v1[4], v2[4], r[4];
+    tip_column(&sP[0][cat][0], s1, v1);
+    tip_column(&sP[1][cat][0], s2, v2);
+#pragma unroll
+    for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+    int e = 0;
+    if (SCALE == 1) {
+      T m = fmax(fmax(r[0], r[1]), fmax(r[2], r[3]));
+#pragma unroll
+      for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+      e = frexp_exp(m);
+      scale_pow2(r, e);
+    }
+    if (t / C < 25) {
+      V4<T>::st(tab + (size_t)t * 4, r);
+      if (cat == 0) tabe[combo] = e;
+    }
+  }
+  consumer_sync();
+}
+
 // Consumer loop over chunks [c0, c1) of one operation, specialised on the
 // operation's shape (tip / internal children, scaling) so the per-item body
 // is branch-free: 2 LDS.128 (or 1 per tip child), the 4x4 mat-vecs from
@@ -412,7 +444,8 @@ template <typename T, int C, int kStages, bool TIP1, bool TIP2, int SCALE>
 __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (&P2)[16],
                                    const T *P1tab, const T *P2tab, BulkStage<T, C> *stages,
                                    uint64_t *full, uint64_t *empty, int c0, int c1, int &i,
-                                   unsigned nitems) {
+                                   unsigned nitems, const T *tab, const int *tabe) {
+  constexpr bool kTab = TIP1 && TIP2 && SCALE != 2;  // whole output from the pair table
   const int cat = threadIdx.x % C;
   T *__restrict__ out = static_cast<T *>(op.out);
   for (int chunk = c0; chunk < c1; ++chunk, ++i) {
@@ -425,6 +458,14 @@ __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (
     for (int j = 0; j < kChunkItems / kThreads; ++j) {  // ---- read the stage
       const int li = threadIdx.x + j * kThreads;
       const int lp = li / C;
+      if constexpr (kTab) {
+        const unsigned s1 = min((unsigned)reinterpret_cast<const uint8_t *>(st.c1)[lp], 4u);
+        const unsigned s2 = min((unsigned)reinterpret_cast<const uint8_t *>(st.c2)[lp], 4u);
+        const int combo = (int)(s1 * 5 + s2);
+        V4<T>::lds(tab + (combo * C + cat) * 4, r[j]);
+        ex[j] = tabe[combo];
+        continue;
+      }
       T v1[4], v2[4];
       if (TIP1) {
         tip_column(P1tab, reinterpret_cast<const uint8_t *>(st.c1)[lp], v1);
@@ -467,7 +508,9 @@ __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (
       const int li = threadIdx.x + j * kThreads;
       const unsigned item = (unsigned)chunk * kChunkItems + li;
       const bool valid = item < nitems;
-      if (SCALE == 1) {
+      if (kTab) {
+        if (SCALE == 1 && valid && cat == 0) op.scale_out[item / C] = ex[j];  // tips: no child exponents
+      } else if (SCALE == 1) {
         T m = fmax(fmax(r[j][0], r[j][1]), fmax(r[j][2], r[j][3]));
 #pragma unroll
         for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
@@ -493,6 +536,8 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
   extern __shared__ __align__(128) unsigned char smem_raw[];
   S *stages = reinterpret_cast<S *>(smem_raw);
   __shared__ __align__(16) T sP[2][C][kPTab];
+  __shared__ __align__(16) T sTab[25 * C * 4];  // tip-tip pair table (build_tiptip_table)
+  __shared__ int sTabE[25];
   __shared__ __align__(8) uint64_t full[kStages];
   __shared__ __align__(8) uint64_t empty[kStages];
 
@@ -542,10 +587,12 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
     const T *P2t = &sP[1][cat][0];
     const int scale = op.scale_out != nullptr ? 1 : (op.scale_in != nullptr ? 2 : 0);
     const int kind = (op.flags & 3) * 3 + scale;
+    if (kind == 9) build_tiptip_table<T, C, 0>(sP, sTab, sTabE);
+    if (kind == 10) build_tiptip_table<T, C, 1>(sP, sTab, sTabE);
 #define RRL_BULK_CASE(K, T1, T2, SC)                                                               \
   case K:                                                                                         \
     bulk_chunks<T, C, kStages, T1, T2, SC>(op, P1, P2, P1t, P2t, stages, full, empty, c0, c1, i,   \
-                                           nitems);                                               \
+                                           nitems, sTab, sTabE);                                  \
     break;
     switch (kind) {
       RRL_BULK_CASE(0, false, false, 0)

@@ -503,6 +503,26 @@ def test_dest_scale_read_reuses_factors(kind, p, model, precision):
     tl.close()
 
 
+@pytest.mark.parametrize("precision", [64, 32])
+def test_unscaled_bulk_pass_with_tip_pairs(precision):
+    """Bulk-path operations with two tip children read their whole output from a
+    per-operation table of the 5 x 5 state pairs (missing included); with no
+    rescaling at all (dest_scale_write = dest_scale_read = -1) the pass must
+    still match the oracle (small tree: nothing underflows)."""
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="yule", n=30, p=20_000, model="gtr", c=4, seed=23, missing_frac=0.1)
+    tl = gpu_setup(w, "reroot", precision, cumulative=False)
+    R.rrl_update_transition_matrices(tl.inst, 0, tl.matrix_idx, tl.t)
+    ops = tl.ops.copy()
+    ops["dest_scale_write"] = -1
+    ops["dest_scale_read"] = -1
+    R.rrl_update_partials(tl.inst, ops, tl.offsets)
+    got = R.rrl_calculate_root_log_likelihoods(tl.inst, tl.root_buffer, 0, 0, tl.n_scale - 1)  # zeros
+    ora = oracle_run(w)
+    assert rel(got, ora.lnl) <= LNL_TOL[precision], (got, ora.lnl)
+    tl.close()
+
+
 # ------------------------------------------------------------------ pattern partitions (NEXT-3)
 @pytest.mark.parametrize("precision,s_model", [(64, "gtr"), (32, "gtr"), (32, "gy94"), (64, "gy94"),
                                                (32, "gtr_bulk"), (64, "gtr_bulk")])
