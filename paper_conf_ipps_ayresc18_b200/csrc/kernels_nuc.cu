@@ -350,9 +350,25 @@ struct BulkStage {
   int32_t e2[kPat];
 };
 
+// Pair-table operations (two tip children, not applying stored factors) move
+// only 1-byte tip codes, so one stage carries up to kTipGroup consecutive
+// chunks of them (one copy per child instead of one per chunk): the producer
+// and the consumers derive the same group sizes from the same arguments.
+constexpr int kTipGroup = 16;
+__device__ inline bool pair_table_op(const DevOp &op) {
+  return (op.flags & (OP_TIP1 | OP_TIP2)) == (OP_TIP1 | OP_TIP2) &&
+         (op.scale_out != nullptr || op.scale_in == nullptr);
+}
+template <int C>
+__device__ inline int tip_group(const DevOp &op, int chunk, int chunk_end) {
+  const int valid = (int)(((long long)op.p * C + kChunkItems - 1) / kChunkItems);  // chunks inside op.p
+  if (chunk >= valid) return 1;
+  return min(kTipGroup, min(chunk_end, valid) - chunk);
+}
+
 // Issue every bulk copy of chunk `chunk` of operation `oi` into `st`, arming `bar`.
 template <typename T, int C>
-__device__ inline void issue_chunk(const DevOp *ops, int oi, int chunk, BulkStage<T, C> *st,
+__device__ inline void issue_chunk(const DevOp *ops, int oi, int chunk, int group, BulkStage<T, C> *st,
                                    uint64_t *bar) {
   using S = BulkStage<T, C>;
   const DevOp &op = ops[oi];
@@ -361,6 +377,14 @@ __device__ inline void issue_chunk(const DevOp *ops, int oi, int chunk, BulkStag
     return;
   }
   const bool t1 = op.flags & OP_TIP1, t2 = op.flags & OP_TIP2;
+  if (pair_table_op(op)) {  // `group` chunks of tip codes
+    const unsigned b = (unsigned)group * S::kPat;
+    mbar_expect_tx(bar, 2 * b);
+    const size_t pat0 = (size_t)chunk * S::kPat;
+    bulk_g2s(st->c1, static_cast<const uint8_t *>(op.in1) + pat0, b, bar);
+    bulk_g2s(st->c2, static_cast<const uint8_t *>(op.in2) + pat0, b, bar);
+    return;
+  }
   const bool cum = op.scale_out != nullptr;
   const bool e1 = cum && !t1 && op.cum1 != nullptr, e2 = cum && !t2 && op.cum2 != nullptr;
   const unsigned b1 = t1 ? S::kPat : S::kPartBytes, b2 = t2 ? S::kPat : S::kPartBytes;
@@ -448,6 +472,33 @@ __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (
   constexpr bool kTab = TIP1 && TIP2 && SCALE != 2;  // whole output from the pair table
   const int cat = threadIdx.x % C;
   T *__restrict__ out = static_cast<T *>(op.out);
+  if constexpr (kTab) {
+    for (int chunk = c0; chunk < c1; ++i) {
+      const int g = tip_group<C>(op, chunk, c1);
+      const int s = i % kStages;
+      mbar_wait(&full[s], (unsigned)(i / kStages) & 1u);
+      const BulkStage<T, C> &st = stages[s];
+      const uint8_t *k1 = reinterpret_cast<const uint8_t *>(st.c1), *k2 = reinterpret_cast<const uint8_t *>(st.c2);
+      for (int q = 0; q < g; ++q) {
+#pragma unroll
+        for (int j = 0; j < kChunkItems / kThreads; ++j) {
+          const int li = threadIdx.x + j * kThreads;
+          const int lp = q * (kChunkItems / C) + li / C;
+          const unsigned item = (unsigned)(chunk + q) * kChunkItems + li;
+          const unsigned combo = min((unsigned)k1[lp], 4u) * 5 + min((unsigned)k2[lp], 4u);
+          T r[4];
+          V4<T>::lds(tab + (combo * C + cat) * 4, r);
+          if (item < nitems) {
+            if (SCALE == 1 && cat == 0) op.scale_out[item / C] = tabe[combo];  // tips: no child exponents
+            V4<T>::st(out + (size_t)item * 4, r);
+          }
+        }
+      }
+      __syncwarp();
+      if ((threadIdx.x & 31) == 0) mbar_arrive(&empty[s]);
+      chunk += g;
+    }
+  } else {
   for (int chunk = c0; chunk < c1; ++chunk, ++i) {
     const int s = i % kStages;
     mbar_wait(&full[s], (unsigned)(i / kStages) & 1u);
@@ -458,14 +509,6 @@ __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (
     for (int j = 0; j < kChunkItems / kThreads; ++j) {  // ---- read the stage
       const int li = threadIdx.x + j * kThreads;
       const int lp = li / C;
-      if constexpr (kTab) {
-        const unsigned s1 = min((unsigned)reinterpret_cast<const uint8_t *>(st.c1)[lp], 4u);
-        const unsigned s2 = min((unsigned)reinterpret_cast<const uint8_t *>(st.c2)[lp], 4u);
-        const int combo = (int)(s1 * 5 + s2);
-        V4<T>::lds(tab + (combo * C + cat) * 4, r[j]);
-        ex[j] = tabe[combo];
-        continue;
-      }
       T v1[4], v2[4];
       if (TIP1) {
         tip_column(P1tab, reinterpret_cast<const uint8_t *>(st.c1)[lp], v1);
@@ -508,9 +551,7 @@ __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (
       const int li = threadIdx.x + j * kThreads;
       const unsigned item = (unsigned)chunk * kChunkItems + li;
       const bool valid = item < nitems;
-      if (kTab) {
-        if (SCALE == 1 && valid && cat == 0) op.scale_out[item / C] = ex[j];  // tips: no child exponents
-      } else if (SCALE == 1) {
+      if (SCALE == 1) {
         T m = fmax(fmax(r[j][0], r[j][1]), fmax(r[j][2], r[j][3]));
 #pragma unroll
         for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
@@ -523,6 +564,7 @@ __device__ inline void bulk_chunks(const DevOp &op, const T (&P1)[16], const T (
       }
       if (valid) V4<T>::st(out + (size_t)item * 4, r[j]);
     }
+  }
   }
 }
 
@@ -558,11 +600,15 @@ k_partials_nuc_bulk(const DevOp *__restrict__ ops, int p, int nchunks, int total
   if (threadIdx.x >= kThreads) {  // ------------------------------ producer warp
     if (threadIdx.x == kThreads) {
       int oi = lo / nchunks, chunk = lo % nchunks;
-      for (int k = 0, f = lo; f < hi; ++f, ++k) {
+      for (int k = 0, f = lo; f < hi; ++k) {
         const int s = k % kStages;
         mbar_wait(&empty[s], ((unsigned)(k / kStages) & 1u) ^ 1u);
-        issue_chunk<T, C>(ops, oi, chunk, &stages[s], &full[s]);
-        if (++chunk == nchunks) { chunk = 0; ++oi; }
+        // the consumers' chunk range of this op ends at min(nchunks, this CTA's end)
+        const int g = pair_table_op(ops[oi]) ? tip_group<C>(ops[oi], chunk, min(nchunks, chunk + (hi - f))) : 1;
+        issue_chunk<T, C>(ops, oi, chunk, g, &stages[s], &full[s]);
+        f += g;
+        chunk += g;
+        if (chunk == nchunks) { chunk = 0; ++oi; }
       }
     }
     return;
