@@ -266,6 +266,8 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-secondary", action="store_true",
                     help="skip the configs[2] HBM-regime measurement that rides along with c1")
+    ap.add_argument("--no-fused", action="store_true",
+                    help="skip the one-launch-per-pass (RRL_FLAG_FUSED_PASS) measurement")
     ap.add_argument("--ref-patterns", type=int, default=10_000)
     args = ap.parse_args()
     args.warmup = max(args.warmup, 3)
@@ -321,13 +323,13 @@ def main():
         allreduce_(t, dist.ReduceOp.MAX)
         return float(t.item())
 
-    def make(w, mode, precision, reuse):
+    def make(w, mode, precision, reuse, fused=False):
         nbuf = None
         if reuse:
             nbuf = R.rrl_reroot_and_schedule(w.n, w.tree.parent, w.tree.blen, mode, True)["buffer_count"]
         tl = TreeLikelihood(w.n, w.p, w.s, w.c, precision=precision, device=local,
                             cuda_graph=not args.no_graph, buffer_count=nbuf,
-                            stream_ptr=stream.cuda_stream)
+                            stream_ptr=stream.cuda_stream, fused_pass=fused)
         tl.set_model_params(w.model, w.rates, w.cat_weights)
         tl.set_tips(w.tips)
         tl.set_pattern_weights(w.pattern_weights)
@@ -443,6 +445,29 @@ def main():
                                  "512 patterns, PAPER.md:258); mean 1.26x (random 256 OTUs, "
                                  "PAPER.md:230)"}
             to.close()
+        if s == 4 and cfg != "c4" and not args.no_fused:
+            # RRL_FLAG_FUSED_PASS (beyond the paper): the whole
+            # pass as ONE launch; level sets still bound its dependent chain.
+            fused = {}
+            for mode in ("reroot", "level"):
+                tf = make(w, mode, precision, False, fused=True)
+                ms_f, prof_f = timed(tf, steps, warmup)
+                pf = maxall(prof_f["partials_ms"]) / nsi
+                fused[mode] = {"value": fl * world * steps / (ms_f * 1e-3) / 1e9,
+                               "ms_per_step": ms_f / steps, "updatePartials_ms_per_pass": pf,
+                               "launches_per_pass": prof_f["partials_launches"] / nsi,
+                               "hbm_gbs": bpp / (pf * 1e-3) / 1e9,
+                               "lnL": float(d_out.item())}
+                tf.close()
+            res["fused_pass"] = {
+                "kernel": "k_partials_nuc_fused (RRL_FLAG_FUSED_PASS: one launch per pass)",
+                "value": fused["reroot"]["value"], "unit": "GFLOPS",
+                "ms_per_step": fused["reroot"]["ms_per_step"],
+                "updatePartials_ms_per_pass": fused["reroot"]["updatePartials_ms_per_pass"],
+                "roofline_frac": fused["reroot"]["hbm_gbs"] / hbm,
+                "reroot_vs_original_updatePartials": fused["level"]["updatePartials_ms_per_pass"]
+                / fused["reroot"]["updatePartials_ms_per_pass"],
+                "original": fused["level"], "lnL": fused["reroot"]["lnL"]}
         if keep:
             res["tl"] = tl
         else:
@@ -519,12 +544,16 @@ def main():
         "clocks": prim["clocks"],
         "lnL": prim["lnL"],
     }
+    if "fused_pass" in prim:
+        out["fused_pass"] = prim["fused_pass"]
     if sec is not None:
         out["hbm_regime"] = {
             "workload": CONFIG_DESC["c2"], "value": sec["value"], "unit": "GFLOPS",
             "ms_per_step": sec["ms_per_step"], "reroot": sec.get("reroot"),
             "updatePartials": sec["updatePartials"], "roofline": sec["roofline"],
             "gpu_launches": int(sec["launches"]), "clocks": sec["clocks"]}
+        if "fused_pass" in sec:
+            out["hbm_regime"]["fused_pass"] = sec["fused_pass"]
     print(json.dumps(out), flush=True)
     if dist is not None:
         dist.destroy_process_group()

@@ -84,6 +84,15 @@ extern "C" {
                                           replay it on later identical calls */
 #define RRL_FLAG_CODON_SIMT 0x4u       /* 61-state fp32: use the FP32 SIMT kernel
                                           instead of the tcgen05 (3xTF32) one */
+#define RRL_FLAG_FUSED_PASS 0x8u       /* 4 states, no pattern ranges: run a whole
+                                          rrl_update_partials call as ONE launch in
+                                          which every thread owns the same (pattern,
+                                          category) items in every operation and
+                                          walks the level sets in order (Eq. (1)
+                                          couples only equal patterns).
+                                          Beyond the paper's one launch per set
+                                          (PAPER.md:116,128); same arithmetic,
+                                          bit-identical results. */
 
 /* Schedule flags (rrl_reroot_and_schedule). Low byte = mode. */
 #define RRL_SCHED_SEQUENTIAL 1u  /* post-order, one op per set (Fig.2 upper) */

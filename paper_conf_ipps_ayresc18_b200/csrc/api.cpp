@@ -807,6 +807,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       }
       I->h_ops[i] = d;
     }
+    for (int k = 0; k < nsets; ++k) I->h_ops[offs[k + 1] - 1].flags |= OP_SET_END;
     CK(cudaMemcpyAsync(I->d_ops, I->h_ops, sizeof(DevOp) * op_count, cudaMemcpyHostToDevice, I->stream));
     CK(cudaEventRecord(I->staging_ev, I->stream));
     I->last_ops.assign(ops, ops + op_count);
@@ -817,7 +818,15 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
     if (rg < 0) return rg;
   }
 
+  const bool fused = I->s == 4 && (I->flags & RRL_FLAG_FUSED_PASS) && !ranges;
   auto launch_all = [&](bool capturing) -> int {
+    if (fused) {  // one launch for every set (RRL_FLAG_FUSED_PASS)
+      Timed tm(I, 0, !capturing);
+      const int e = launch_update_partials_nuc_fused(I->prec, I->c, I->d_ops, op_count, I->p, I->stream);
+      if (e != 0) return fail(RRL_ERROR_CUDA, std::string("updatePartials fused launch: ") +
+                                                  cudaGetErrorString(static_cast<cudaError_t>(e)));
+      return 0;
+    }
     for (int k = 0; k < nsets; ++k) {
       const int n = offs[k + 1] - offs[k];
       int pmax = I->p;  // widest pattern range of the set (grids are sized for it)
@@ -850,7 +859,9 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
     return 0;
   };
   int kl = 0;
-  for (int k = 0; k < nsets; ++k) kl += (offs[k + 1] - offs[k] + 65534) / 65535;
+  if (fused) kl = 1;
+  else
+    for (int k = 0; k < nsets; ++k) kl += (offs[k + 1] - offs[k] + 65534) / 65535;
 
   // (the legacy default stream cannot be captured: eager launches there)
   const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && I->stream != nullptr;

@@ -31,6 +31,7 @@
 // + c x 4 x sizeof(T) out + exponents; 1.8 flop/B in fp32.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 
 #include "rrl_internal.h"
@@ -309,6 +310,89 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 #pragma unroll
       for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
       finish_item<T, C>(op, r, valid, pat, cat, ca[j], cb[j], out + (size_t)item * 4);
+    }
+  }
+}
+
+// ============================================================ fused pass
+// RRL_FLAG_FUSED_PASS (beyond the paper): the whole operation
+// list in ONE launch.  Eq. (1) couples a pattern's partials only to the same
+// pattern of the children, and every operation maps item
+// (pattern, category) to the same thread here, so each thread's inputs in
+// level set k are its own outputs of earlier sets: program order replaces the
+// launch boundary, no grid or block synchronisation is needed.  Level sets
+// still bound the dependent chain: the G operations of a group (one set) issue
+// all their reads together, so a pass costs ~one memory round trip per set
+// (rerooting keeps its effect) instead of one launch per set.  Reads of
+// partials / exponents written in this launch are plain coherent loads (no
+// __ldg); transition matrices and tip states were written before it.
+template <typename T, int C, int G>
+__global__ void __launch_bounds__(kThreads)
+k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks) {
+  const int cat = threadIdx.x % C;
+  const unsigned nitems = (unsigned)p * C;
+  pdl_wait();
+  for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
+    const unsigned item = (unsigned)chunk * kThreads + threadIdx.x;
+    const bool valid = item < nitems;
+    const unsigned pat = valid ? item / C : 0u;
+    for (int i = 0; i < nops;) {
+      int ng = 1;  // ops of this group: consecutive, within one level set
+      while (ng < G && i + ng < nops && !(ops[i + ng - 1].flags & OP_SET_END)) ++ng;
+      T P1[G][16], P2[G][16], L1[G][4], L2[G][4];
+      unsigned s1[G], s2[G];
+      int ca[G], cb[G];
+#pragma unroll
+      for (int j = 0; j < G; ++j) {  // ---- every read of the group in flight together
+        if (j < ng) {
+          const DevOp &op = ops[i + j];
+          const bool sw = op.scale_out != nullptr;
+#pragma unroll
+          for (int k = 0; k < 16; k += 4) {
+            V4<T>::ld(static_cast<const T *>(op.P1) + cat * 16 + k, *reinterpret_cast<T(*)[4]>(&P1[j][k]));
+            V4<T>::ld(static_cast<const T *>(op.P2) + cat * 16 + k, *reinterpret_cast<T(*)[4]>(&P2[j][k]));
+          }
+          s1[j] = s2[j] = 4u;
+#pragma unroll
+          for (int z = 0; z < 4; ++z) L1[j][z] = L2[j][z] = T(0);
+          if (op.flags & OP_TIP1) {
+            if (valid) s1[j] = __ldg(static_cast<const uint8_t *>(op.in1) + pat);
+          } else if (valid) {
+            V4<T>::lds(static_cast<const T *>(op.in1) + (size_t)item * 4, L1[j]);
+          }
+          if (op.flags & OP_TIP2) {
+            if (valid) s2[j] = __ldg(static_cast<const uint8_t *>(op.in2) + pat);
+          } else if (valid) {
+            V4<T>::lds(static_cast<const T *>(op.in2) + (size_t)item * 4, L2[j]);
+          }
+          ca[j] = (sw && valid && cat == 0 && op.cum1 != nullptr) ? op.cum1[pat] : 0;
+          cb[j] = (sw && valid && cat == 0 && op.cum2 != nullptr) ? op.cum2[pat] : 0;
+        }
+      }
+#pragma unroll
+      for (int j = 0; j < G; ++j) {  // ---- compute, rescale, store
+        if (j < ng) {
+          const DevOp &op = ops[i + j];
+          T v1[4], v2[4], r[4];
+          if (op.flags & OP_TIP1) tip_select(P1[j], s1[j], v1); else matvec_r(P1[j], L1[j], v1);
+          if (op.flags & OP_TIP2) tip_select(P2[j], s2[j], v2); else matvec_r(P2[j], L2[j], v2);
+#pragma unroll
+          for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+          if (op.scale_out != nullptr) {
+            T m = valid ? fmax(fmax(r[0], r[1]), fmax(r[2], r[3])) : T(0);
+#pragma unroll
+            for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+            const int e = frexp_exp(m);
+            if (e != 0) scale_pow2(r, e);
+            if (valid && cat == 0) op.scale_out[pat] = e + ca[j] + cb[j];
+          } else if (op.scale_in != nullptr) {
+            const int e = valid ? op.scale_in[pat] : 0;
+            if (e != 0) scale_pow2(r, e);
+          }
+          if (valid) V4<T>::st(static_cast<T *>(op.out) + (size_t)item * 4, r);
+        }
+      }
+      i += ng;
     }
   }
 }
@@ -766,7 +850,49 @@ int dispatch_c(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p, i
   }
 }
 
+template <typename T, int C>
+int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
+  constexpr int G = 2;
+  static int resident = -1;  // per template instance
+  if (resident < 0) {
+    int per_sm = 1, dev = 0, nsm = 148;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G>, kThreads, 0);
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    resident = (per_sm > 0 ? per_sm : 1) * nsm;
+  }
+  const long long items = (long long)p * C;
+  const int nchunks = (int)((items + kThreads - 1) / kThreads);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)std::min(nchunks, resident));
+  cfg.blockDim = dim3(kThreads);
+  cfg.stream = st;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  at[0].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_fused<T, C, G>, d_ops, nops, p, nchunks);
+}
+
+template <typename T>
+int dispatch_fused(int c, const DevOp *d_ops, int nops, int p, cudaStream_t st) {
+  switch (c) {
+    case 1: return launch_fused_t<T, 1>(d_ops, nops, p, st);
+    case 2: return launch_fused_t<T, 2>(d_ops, nops, p, st);
+    case 4: return launch_fused_t<T, 4>(d_ops, nops, p, st);
+    case 8: return launch_fused_t<T, 8>(d_ops, nops, p, st);
+    default: return (int)cudaErrorInvalidValue;
+  }
+}
+
 }  // namespace
+
+int launch_update_partials_nuc_fused(int prec, int c, const DevOp *d_ops, int nops, int p, void *stream) {
+  if (nops <= 0 || p <= 0) return 0;
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  return prec == 32 ? dispatch_fused<float>(c, d_ops, nops, p, st) : dispatch_fused<double>(c, d_ops, nops, p, st);
+}
 
 int launch_update_partials_nuc(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
                                int p, int /*p_pad*/, int early, void *stream) {

@@ -35,7 +35,8 @@ struct DevOp {
 };
 static_assert(sizeof(DevOp) == 104, "DevOp layout");
 
-enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2 };
+// OP_SET_END marks the last operation of a level set (read by the fused-pass kernel).
+enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2, OP_SET_END = 4 };
 
 // ---------------------------------------------------------------- launchers
 // All launchers enqueue on `stream` and return cudaError_t as int.
@@ -43,6 +44,9 @@ enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2 };
 // (small sets are passed by value in the kernel parameters), may be null.
 int launch_update_partials_nuc(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
                                int p, int p_pad, int early, void *stream);
+// RRL_FLAG_FUSED_PASS: the whole 4-state operation list (sets marked by
+// OP_SET_END, no pattern ranges) as one launch.
+int launch_update_partials_nuc_fused(int prec, int c, const DevOp *d_ops, int nops, int p, void *stream);
 int launch_update_partials_codon(int prec, int c, const DevOp *d_ops, const DevOp *h_ops, int nops,
                                  int p, int p_pad, void *stream);
 // tcgen05 (tf32, 3xTF32) codon kernel: fp32, c in {1,2,4,8}; cudaErrorNotSupported otherwise.

@@ -38,13 +38,14 @@ class TreeLikelihood:
     def __init__(self, n: int, p: int, s: int, c: int, precision: int = 32, device: int = 0,
                  cumulative_scaling: bool = True, cuda_graph: bool = False,
                  buffer_count: int | None = None, stream_ptr: int | None = None,
-                 codon_simt: bool = False, partitions: int = 1):
+                 codon_simt: bool = False, partitions: int = 1, fused_pass: bool = False):
         self.n, self.p, self.s, self.c, self.precision = n, p, s, c, precision
         self.cumulative = cumulative_scaling
         nbuf = buffer_count if buffer_count is not None else 2 * n - 1
         n_scale = nbuf - n + (0 if cumulative_scaling else 1)
         flags = (R.FLAG_SCALE_CUMULATIVE if cumulative_scaling else 0) | \
-                (R.FLAG_CUDA_GRAPH if cuda_graph else 0) | (R.FLAG_CODON_SIMT if codon_simt else 0)
+                (R.FLAG_CUDA_GRAPH if cuda_graph else 0) | (R.FLAG_CODON_SIMT if codon_simt else 0) | \
+                (R.FLAG_FUSED_PASS if fused_pass else 0)
         self.nbuf = nbuf
         self.n_scale = n_scale
         self.partitions = partitions

@@ -36,6 +36,7 @@ NONE = -1
 FLAG_SCALE_CUMULATIVE = 0x1
 FLAG_CUDA_GRAPH = 0x2
 FLAG_CODON_SIMT = 0x4
+FLAG_FUSED_PASS = 0x8
 SCHED_SEQUENTIAL = 1
 SCHED_LEVEL = 2
 SCHED_REROOT = 3

@@ -14,7 +14,7 @@ def oracle_run(w, tree=None, keep_partials=False):
 
 
 def gpu_setup(w, mode="reroot", precision=64, cumulative=True, graph=False, reuse=False,
-              tree=None, codon_simt=False):
+              tree=None, codon_simt=False, fused=False):
     from paper_conf_ipps_ayresc18_b200 import TreeLikelihood
     t = tree if tree is not None else w.tree
     nbuf = None
@@ -22,7 +22,8 @@ def gpu_setup(w, mode="reroot", precision=64, cumulative=True, graph=False, reus
         from paper_conf_ipps_ayresc18_b200 import rrl as R
         nbuf = R.rrl_reroot_and_schedule(t.n, t.parent, t.blen, mode, True)["buffer_count"]
     tl = TreeLikelihood(w.n, w.p, w.s, w.c, precision=precision, cumulative_scaling=cumulative,
-                        cuda_graph=graph, buffer_count=nbuf, codon_simt=codon_simt)
+                        cuda_graph=graph, buffer_count=nbuf, codon_simt=codon_simt,
+                        fused_pass=fused)
     tl.set_model_params(w.model, w.rates, w.cat_weights)
     tl.set_tips(w.tips)
     tl.set_pattern_weights(w.pattern_weights)

@@ -564,3 +564,53 @@ def test_pattern_partitions_one_launch_per_set(precision, s_model):
         sub.pattern_weights = np.ones(e - b)
         assert rel(got[k], oracle_run(sub).lnl) <= LNL_TOL[precision], k
     tl.close()
+
+
+# ------------------------------------------------------------------ fused pass (RRL_FLAG_FUSED_PASS)
+FUSED_CASES = [  # (kind, n, p, c, precision, mode, cumulative, reuse)
+    ("pectinate", 128, 10_000, 4, 32, "reroot", True, False),    # configs[1]
+    ("pectinate", 128, 10_000, 4, 32, "level", True, False),
+    ("pectinate", 128, 10_000, 4, 64, "reroot", True, False),
+    ("yule", 300, 777, 4, 32, "reroot", True, False),
+    ("yule", 300, 777, 4, 64, "sequential", True, False),
+    ("random", 64, 1_001, 1, 32, "reroot", False, False),
+    ("random", 64, 1_001, 2, 64, "reroot", False, False),
+    ("random", 90, 3_333, 8, 32, "reroot", True, False),
+    ("pectinate", 500, 2_000, 4, 32, "reroot", True, True),     # liveness buffer reuse
+    ("yule", 40, 17_001, 4, 64, "reroot", True, False),        # bulk path when not fused
+    ("random", 3, 5, 4, 32, "reroot", True, False),
+    ("random", 2, 1, 4, 64, "reroot", True, False),
+]
+
+
+@pytest.mark.parametrize("kind,n,p,c,precision,mode,cumulative,reuse", FUSED_CASES)
+def test_fused_pass_bit_identical_to_level_sets(kind, n, p, c, precision, mode, cumulative, reuse):
+    """One launch per pass (each thread owns its items across all level sets)
+    gives the per-set launches' results bit for bit, and the oracle's lnL."""
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind=kind, n=n, p=p, model="gtr", c=c, seed=n + p + c, missing_frac=0.05)
+    a = gpu_setup(w, mode, precision, cumulative=cumulative, reuse=reuse)
+    b = gpu_setup(w, mode, precision, cumulative=cumulative, reuse=reuse, fused=True)
+    la, lb = a.loglik(), b.loglik()
+    assert la == lb, (la, lb)
+    assert rel(lb, oracle_run(w).lnl) <= LNL_TOL[precision]
+    if not reuse:
+        for v in range(n, 2 * n - 1):
+            np.testing.assert_array_equal(a.partials(v), b.partials(v))
+    for k in range(b.n_scale):
+        np.testing.assert_array_equal(a.scale(k), b.scale(k))
+    R.rrl_reset_profile(b.inst)
+    b.loglik()
+    assert R.rrl_get_profile(b.inst)["partials_launches"] == 1
+    a.close()
+    b.close()
+
+
+def test_fused_pass_graph_replay():
+    w = make_workload(tree_kind="yule", n=150, p=4_000, model="gtr", c=4, seed=5)
+    a = gpu_setup(w, "reroot", 32)
+    g = gpu_setup(w, "reroot", 32, graph=True, fused=True)
+    ref = a.loglik()
+    assert g.loglik() == ref and g.loglik() == ref         # capture, then replay
+    a.close()
+    g.close()
