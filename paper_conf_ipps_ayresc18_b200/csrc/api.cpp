@@ -808,6 +808,25 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       I->h_ops[i] = d;
     }
     for (int k = 0; k < nsets; ++k) I->h_ops[offs[k + 1] - 1].flags |= OP_SET_END;
+    // fused pass: children produced by one of the previous W-1 ops are read
+    // from the thread's shared-memory ring (slot = producer index mod W)
+    const int W = fused_ring(I->prec);
+    for (int i = 0; i < op_count; ++i) {
+      DevOp &d = I->h_ops[i];
+      int32_t *ring[2] = {&d.ring1, &d.ring2};
+      const int ch[2] = {ops[i].child1, ops[i].child2};
+      const int32_t *cum[2] = {d.cum1, d.cum2};
+      for (int b = 0; b < 2; ++b) {
+        *ring[b] = -1;
+        if (d.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) continue;
+        for (int j = i - 1; j >= 0 && j > i - W; --j) {
+          if (ops[j].dest != ch[b]) continue;
+          *ring[b] = j % W;
+          if (cum[b] != nullptr && I->h_ops[j].scale_out == cum[b]) d.flags |= (b == 0 ? OP_RING_E1 : OP_RING_E2);
+          break;
+        }
+      }
+    }
     CK(cudaMemcpyAsync(I->d_ops, I->h_ops, sizeof(DevOp) * op_count, cudaMemcpyHostToDevice, I->stream));
     CK(cudaEventRecord(I->staging_ev, I->stream));
     I->last_ops.assign(ops, ops + op_count);

@@ -323,12 +323,20 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 // launch boundary, no grid or block synchronisation is needed.  Level sets
 // still bound the dependent chain: the G operations of a group (one set) issue
 // all their reads together, so a pass costs ~one memory round trip per set
-// (rerooting keeps its effect) instead of one launch per set.  Reads of
+// (rerooting keeps its effect) instead of one launch per set.  A child made
+// by one of the previous W-1 operations comes from the thread's own slot of a
+// shared-memory ring (host-resolved DevOp::ring1/ring2), so on a rerooted
+// pectinate tree the chain never leaves the SM.  Other reads of
 // partials / exponents written in this launch are plain coherent loads (no
 // __ldg); transition matrices and tip states were written before it.
-template <typename T, int C, int G>
+template <typename T, int C, int G, int W>
 __global__ void __launch_bounds__(kThreads)
 k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks) {
+  // per-thread ring of the last W operations' outputs (and cumulative
+  // exponents): a child produced by one of the previous W-1 ops is read back
+  // from shared memory, off the L2 round trip (DevOp::ring1/ring2)
+  __shared__ __align__(16) T ringL[W][kThreads][4];
+  __shared__ int ringE[W][kThreads];
   const int cat = threadIdx.x % C;
   const unsigned nitems = (unsigned)p * C;
   pdl_wait();
@@ -355,18 +363,23 @@ k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks
           s1[j] = s2[j] = 4u;
 #pragma unroll
           for (int z = 0; z < 4; ++z) L1[j][z] = L2[j][z] = T(0);
-          if (op.flags & OP_TIP1) {
+          const int fl = op.flags, r1 = op.ring1, r2 = op.ring2;
+          if (fl & OP_TIP1) {
             if (valid) s1[j] = __ldg(static_cast<const uint8_t *>(op.in1) + pat);
           } else if (valid) {
-            V4<T>::lds(static_cast<const T *>(op.in1) + (size_t)item * 4, L1[j]);
+            V4<T>::lds(r1 >= 0 ? &ringL[r1][threadIdx.x][0] : static_cast<const T *>(op.in1) + (size_t)item * 4,
+                       L1[j]);
           }
-          if (op.flags & OP_TIP2) {
+          if (fl & OP_TIP2) {
             if (valid) s2[j] = __ldg(static_cast<const uint8_t *>(op.in2) + pat);
           } else if (valid) {
-            V4<T>::lds(static_cast<const T *>(op.in2) + (size_t)item * 4, L2[j]);
+            V4<T>::lds(r2 >= 0 ? &ringL[r2][threadIdx.x][0] : static_cast<const T *>(op.in2) + (size_t)item * 4,
+                       L2[j]);
           }
-          ca[j] = (sw && valid && cat == 0 && op.cum1 != nullptr) ? op.cum1[pat] : 0;
-          cb[j] = (sw && valid && cat == 0 && op.cum2 != nullptr) ? op.cum2[pat] : 0;
+          ca[j] = (sw && valid && cat == 0 && op.cum1 != nullptr)
+                      ? ((fl & OP_RING_E1) ? ringE[r1][threadIdx.x] : op.cum1[pat]) : 0;
+          cb[j] = (sw && valid && cat == 0 && op.cum2 != nullptr)
+                      ? ((fl & OP_RING_E2) ? ringE[r2][threadIdx.x] : op.cum2[pat]) : 0;
         }
       }
 #pragma unroll
@@ -378,17 +391,21 @@ k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks
           if (op.flags & OP_TIP2) tip_select(P2[j], s2[j], v2); else matvec_r(P2[j], L2[j], v2);
 #pragma unroll
           for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+          const int slot = (i + j) % W;
           if (op.scale_out != nullptr) {
             T m = valid ? fmax(fmax(r[0], r[1]), fmax(r[2], r[3])) : T(0);
 #pragma unroll
             for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
             const int e = frexp_exp(m);
             if (e != 0) scale_pow2(r, e);
-            if (valid && cat == 0) op.scale_out[pat] = e + ca[j] + cb[j];
+            const int et = e + ca[j] + cb[j];
+            ringE[slot][threadIdx.x] = et;
+            if (valid && cat == 0) op.scale_out[pat] = et;
           } else if (op.scale_in != nullptr) {
             const int e = valid ? op.scale_in[pat] : 0;
             if (e != 0) scale_pow2(r, e);
           }
+          V4<T>::st(&ringL[slot][threadIdx.x][0], r);
           if (valid) V4<T>::st(static_cast<T *>(op.out) + (size_t)item * 4, r);
         }
       }
@@ -853,10 +870,11 @@ int dispatch_c(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p, i
 template <typename T, int C>
 int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   constexpr int G = 2;
+  constexpr int W = fused_ring(sizeof(T) == 4 ? 32 : 64);
   static int resident = -1;  // per template instance
   if (resident < 0) {
     int per_sm = 1, dev = 0, nsm = 148;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G, W>, kThreads, 0);
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     resident = (per_sm > 0 ? per_sm : 1) * nsm;
@@ -872,7 +890,7 @@ int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_fused<T, C, G>, d_ops, nops, p, nchunks);
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_fused<T, C, G, W>, d_ops, nops, p, nchunks);
 }
 
 template <typename T>

@@ -32,11 +32,20 @@ struct DevOp {
   int32_t mat1, mat2;       // transition-matrix indices
   int32_t pat0;             // first pattern of the range
   int32_t bufd;             // dest internal-buffer index in the partials slab
+  // fused pass (4 states): ring slot (op index mod fused_ring(prec)) holding the
+  // child's partials in shared memory if its producer is one of the previous
+  // fused_ring - 1 operations, else -1
+  int32_t ring1, ring2;
 };
-static_assert(sizeof(DevOp) == 104, "DevOp layout");
+static_assert(sizeof(DevOp) == 112, "DevOp layout");
+
+// Fused-pass ring depth (operations whose outputs each thread keeps in shared memory).
+constexpr int fused_ring(int prec) { return prec == 32 ? 8 : 4; }
 
 // OP_SET_END marks the last operation of a level set (read by the fused-pass kernel).
-enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2, OP_SET_END = 4 };
+// OP_RING_E1/2: the child's cumulative exponent is in the ring too (its
+// producer wrote the scale buffer this op reads as cum1/cum2).
+enum : int32_t { OP_TIP1 = 1, OP_TIP2 = 2, OP_SET_END = 4, OP_RING_E1 = 8, OP_RING_E2 = 16 };
 
 // ---------------------------------------------------------------- launchers
 // All launchers enqueue on `stream` and return cudaError_t as int.
