@@ -329,87 +329,129 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 // pectinate tree the chain never leaves the SM.  Other reads of
 // partials / exponents written in this launch are plain coherent loads (no
 // __ldg); transition matrices and tip states were written before it.
+// Shared-memory layout of the fused kernel: the ring, then one window of
+// descriptors, their transition matrices [op][branch][cat][16] and their tip
+// codes [op][branch][pattern of the chunk].
+template <typename T, int C, int W> struct FusedSmem {
+  static constexpr int kPats = kThreads / C;  // patterns per chunk
+  static constexpr size_t ring = (size_t)W * kThreads * (4 * sizeof(T) + sizeof(int));
+  static constexpr size_t per_op = sizeof(DevOp) + 2 * C * 16 * sizeof(T) + 2 * kPats;
+  static size_t bytes(int wops) { return ring + (size_t)wops * per_op; }
+};
+
 template <typename T, int C, int G, int W>
 __global__ void __launch_bounds__(kThreads)
-k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks) {
+k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks, int wops) {
+  using S = FusedSmem<T, C, W>;
+  extern __shared__ __align__(16) unsigned char fsm[];
   // per-thread ring of the last W operations' outputs (and cumulative
   // exponents): a child produced by one of the previous W-1 ops is read back
   // from shared memory, off the L2 round trip (DevOp::ring1/ring2)
-  __shared__ __align__(16) T ringL[W][kThreads][4];
-  __shared__ int ringE[W][kThreads];
+  T (*ringL)[kThreads][4] = reinterpret_cast<T (*)[kThreads][4]>(fsm);
+  int (*ringE)[kThreads] = reinterpret_cast<int (*)[kThreads]>(fsm + (size_t)W * kThreads * 4 * sizeof(T));
+  DevOp *sOps = reinterpret_cast<DevOp *>(fsm + S::ring);
+  T *sP = reinterpret_cast<T *>(fsm + S::ring + (size_t)wops * sizeof(DevOp));
+  uint8_t *sTip = reinterpret_cast<uint8_t *>(sP + (size_t)wops * 2 * C * 16);
   const int cat = threadIdx.x % C;
+  const int lpat = threadIdx.x / C;
   const unsigned nitems = (unsigned)p * C;
   pdl_wait();
   for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
     const unsigned item = (unsigned)chunk * kThreads + threadIdx.x;
     const bool valid = item < nitems;
     const unsigned pat = valid ? item / C : 0u;
-    for (int i = 0; i < nops;) {
-      int ng = 1;  // ops of this group: consecutive, within one level set
-      while (ng < G && i + ng < nops && !(ops[i + ng - 1].flags & OP_SET_END)) ++ng;
-      T P1[G][16], P2[G][16], L1[G][4], L2[G][4];
-      unsigned s1[G], s2[G];
-      int ca[G], cb[G];
-#pragma unroll
-      for (int j = 0; j < G; ++j) {  // ---- every read of the group in flight together
-        if (j < ng) {
-          const DevOp &op = ops[i + j];
-          const bool sw = op.scale_out != nullptr;
-#pragma unroll
-          for (int k = 0; k < 16; k += 4) {
-            V4<T>::ld(static_cast<const T *>(op.P1) + cat * 16 + k, *reinterpret_cast<T(*)[4]>(&P1[j][k]));
-            V4<T>::ld(static_cast<const T *>(op.P2) + cat * 16 + k, *reinterpret_cast<T(*)[4]>(&P2[j][k]));
-          }
-          s1[j] = s2[j] = 4u;
-#pragma unroll
-          for (int z = 0; z < 4; ++z) L1[j][z] = L2[j][z] = T(0);
-          const int fl = op.flags, r1 = op.ring1, r2 = op.ring2;
-          if (fl & OP_TIP1) {
-            if (valid) s1[j] = __ldg(static_cast<const uint8_t *>(op.in1) + pat);
-          } else if (valid) {
-            V4<T>::lds(r1 >= 0 ? &ringL[r1][threadIdx.x][0] : static_cast<const T *>(op.in1) + (size_t)item * 4,
-                       L1[j]);
-          }
-          if (fl & OP_TIP2) {
-            if (valid) s2[j] = __ldg(static_cast<const uint8_t *>(op.in2) + pat);
-          } else if (valid) {
-            V4<T>::lds(r2 >= 0 ? &ringL[r2][threadIdx.x][0] : static_cast<const T *>(op.in2) + (size_t)item * 4,
-                       L2[j]);
-          }
-          ca[j] = (sw && valid && cat == 0 && op.cum1 != nullptr)
-                      ? ((fl & OP_RING_E1) ? ringE[r1][threadIdx.x] : op.cum1[pat]) : 0;
-          cb[j] = (sw && valid && cat == 0 && op.cum2 != nullptr)
-                      ? ((fl & OP_RING_E2) ? ringE[r2][threadIdx.x] : op.cum2[pat]) : 0;
-        }
+    for (int w0 = 0; w0 < nops; w0 += wops) {
+      // ---- stage the window: descriptors, then (one round trip) every
+      // matrix and tip code of its ops; none depends on partials
+      const int nw = min(wops, nops - w0);
+      __syncthreads();  // the previous window is consumed
+      {
+        const int4 *src = reinterpret_cast<const int4 *>(ops + w0);
+        int4 *dst = reinterpret_cast<int4 *>(sOps);
+        for (int t = threadIdx.x; t < nw * (int)(sizeof(DevOp) / 16); t += kThreads) dst[t] = __ldg(src + t);
       }
-#pragma unroll
-      for (int j = 0; j < G; ++j) {  // ---- compute, rescale, store
-        if (j < ng) {
-          const DevOp &op = ops[i + j];
-          T v1[4], v2[4], r[4];
-          if (op.flags & OP_TIP1) tip_select(P1[j], s1[j], v1); else matvec_r(P1[j], L1[j], v1);
-          if (op.flags & OP_TIP2) tip_select(P2[j], s2[j], v2); else matvec_r(P2[j], L2[j], v2);
-#pragma unroll
-          for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
-          const int slot = (i + j) % W;
-          if (op.scale_out != nullptr) {
-            T m = valid ? fmax(fmax(r[0], r[1]), fmax(r[2], r[3])) : T(0);
-#pragma unroll
-            for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
-            const int e = frexp_exp(m);
-            if (e != 0) scale_pow2(r, e);
-            const int et = e + ca[j] + cb[j];
-            ringE[slot][threadIdx.x] = et;
-            if (valid && cat == 0) op.scale_out[pat] = et;
-          } else if (op.scale_in != nullptr) {
-            const int e = valid ? op.scale_in[pat] : 0;
-            if (e != 0) scale_pow2(r, e);
-          }
-          V4<T>::st(&ringL[slot][threadIdx.x][0], r);
-          if (valid) V4<T>::st(static_cast<T *>(op.out) + (size_t)item * 4, r);
-        }
+      __syncthreads();
+      constexpr int kV = 16 / sizeof(T);              // elements per 16-byte vector
+      constexpr int kPv = C * 16 / kV;                // vectors per branch
+      for (int t = threadIdx.x; t < nw * 2 * kPv; t += kThreads) {
+        const int o = t / (2 * kPv), r = t % (2 * kPv), br = r / kPv, v = r % kPv;
+        const int4 *src = reinterpret_cast<const int4 *>(br == 0 ? sOps[o].P1 : sOps[o].P2);
+        reinterpret_cast<int4 *>(sP)[t] = __ldg(src + v);
       }
-      i += ng;
+      const unsigned pat0 = (unsigned)chunk * S::kPats;
+      for (int t = threadIdx.x; t < nw * 2 * S::kPats; t += kThreads) {
+        const int o = t / (2 * S::kPats), r = t % (2 * S::kPats), br = r / S::kPats, q = r % S::kPats;
+        const DevOp &op = sOps[o];
+        uint8_t code = 4u;
+        if ((op.flags & (br == 0 ? OP_TIP1 : OP_TIP2)) && pat0 + q < (unsigned)p)
+          code = __ldg(static_cast<const uint8_t *>(br == 0 ? op.in1 : op.in2) + pat0 + q);
+        sTip[t] = code;
+      }
+      __syncthreads();
+      for (int i = w0; i < w0 + nw;) {
+        int ng = 1;  // ops of this group: consecutive, within one level set and window
+        while (ng < G && i + ng < w0 + nw && !(sOps[i + ng - 1 - w0].flags & OP_SET_END)) ++ng;
+        T P1[G][16], P2[G][16], L1[G][4], L2[G][4];
+        unsigned s1[G], s2[G];
+        int ca[G], cb[G];
+#pragma unroll
+        for (int j = 0; j < G; ++j) {  // ---- every read of the group in flight together
+          if (j < ng) {
+            const int o = i + j - w0;
+            const DevOp &op = sOps[o];
+            const bool sw = op.scale_out != nullptr;
+            const T *pt = sP + (size_t)o * 2 * C * 16 + cat * 16;
+#pragma unroll
+            for (int k = 0; k < 16; k += 4) {
+              V4<T>::lds(pt + k, *reinterpret_cast<T(*)[4]>(&P1[j][k]));
+              V4<T>::lds(pt + C * 16 + k, *reinterpret_cast<T(*)[4]>(&P2[j][k]));
+            }
+            s1[j] = sTip[(o * 2 + 0) * S::kPats + lpat];
+            s2[j] = sTip[(o * 2 + 1) * S::kPats + lpat];
+#pragma unroll
+            for (int z = 0; z < 4; ++z) L1[j][z] = L2[j][z] = T(0);
+            const int fl = op.flags, r1 = op.ring1, r2 = op.ring2;
+            if (!(fl & OP_TIP1) && valid)
+              V4<T>::lds(r1 >= 0 ? &ringL[r1][threadIdx.x][0] : static_cast<const T *>(op.in1) + (size_t)item * 4,
+                         L1[j]);
+            if (!(fl & OP_TIP2) && valid)
+              V4<T>::lds(r2 >= 0 ? &ringL[r2][threadIdx.x][0] : static_cast<const T *>(op.in2) + (size_t)item * 4,
+                         L2[j]);
+            ca[j] = (sw && valid && cat == 0 && op.cum1 != nullptr)
+                        ? ((fl & OP_RING_E1) ? ringE[r1][threadIdx.x] : op.cum1[pat]) : 0;
+            cb[j] = (sw && valid && cat == 0 && op.cum2 != nullptr)
+                        ? ((fl & OP_RING_E2) ? ringE[r2][threadIdx.x] : op.cum2[pat]) : 0;
+          }
+        }
+#pragma unroll
+        for (int j = 0; j < G; ++j) {  // ---- compute, rescale, store
+          if (j < ng) {
+            const DevOp &op = sOps[i + j - w0];
+            T v1[4], v2[4], r[4];
+            if (op.flags & OP_TIP1) tip_select(P1[j], s1[j], v1); else matvec_r(P1[j], L1[j], v1);
+            if (op.flags & OP_TIP2) tip_select(P2[j], s2[j], v2); else matvec_r(P2[j], L2[j], v2);
+#pragma unroll
+            for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+            const int slot = (i + j) % W;
+            if (op.scale_out != nullptr) {
+              T m = valid ? fmax(fmax(r[0], r[1]), fmax(r[2], r[3])) : T(0);
+#pragma unroll
+              for (int o = 1; o < C; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
+              const int e = frexp_exp(m);
+              if (e != 0) scale_pow2(r, e);
+              const int et = e + ca[j] + cb[j];
+              ringE[slot][threadIdx.x] = et;
+              if (valid && cat == 0) op.scale_out[pat] = et;
+            } else if (op.scale_in != nullptr) {
+              const int e = valid ? op.scale_in[pat] : 0;
+              if (e != 0) scale_pow2(r, e);
+            }
+            V4<T>::st(&ringL[slot][threadIdx.x][0], r);
+            if (valid) V4<T>::st(static_cast<T *>(op.out) + (size_t)item * 4, r);
+          }
+        }
+        i += ng;
+      }
     }
   }
 }
@@ -871,26 +913,37 @@ template <typename T, int C>
 int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   constexpr int G = 2;
   constexpr int W = fused_ring(sizeof(T) == 4 ? 32 : 64);
-  static int resident = -1;  // per template instance
-  if (resident < 0) {
-    int per_sm = 1, dev = 0, nsm = 148;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G, W>, kThreads, 0);
+  using S = FusedSmem<T, C, W>;
+  constexpr size_t kBudget = 200 * 1024;
+  constexpr int kMaxWin = (int)((kBudget - S::ring) / S::per_op);
+  static_assert(kMaxWin >= 16, "fused window");
+  static int nsm = 0;
+  if (nsm == 0) {
+    cudaError_t e = cudaFuncSetAttribute(k_partials_nuc_fused<T, C, G, W>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBudget);
+    if (e != cudaSuccess) return (int)e;
+    int dev = 0;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    resident = (per_sm > 0 ? per_sm : 1) * nsm;
   }
+  const int wops = std::min(nops, kMaxWin);
+  const size_t smem = S::bytes(wops);
+  int per_sm = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G, W>, kThreads, smem);
+  const int resident = std::max(per_sm, 1) * nsm;
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads - 1) / kThreads);
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3((unsigned)std::min(nchunks, resident));
   cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute at[1];
   at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_fused<T, C, G, W>, d_ops, nops, p, nchunks);
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_fused<T, C, G, W>, d_ops, nops, p, nchunks, wops);
 }
 
 template <typename T>

@@ -12,5 +12,5 @@ python tools/ncu_summary.py $O/prof_fused.ncu-rep c1_fused > $O/ncu_full_c1_fuse
 ncu -i $O/prof_fused.ncu-rep --page raw --csv > $O/ncu_raw_c1_fused.csv 2>/dev/null
 ncu -i $O/prof_fused.ncu-rep --page source --csv > $O/ncu_source_c1_fused.csv 2>/dev/null
 rm -f $O/*.ncu-rep
-timeout 1200 python -m pytest tests -m gpu -q > $O/gpu_tests_full.log 2>&1; tail -3 $O/gpu_tests_full.log
+[ -n "$FULL" ] && timeout 1200 python -m pytest tests -m gpu -q > $O/gpu_tests_full.log 2>&1
 ls -la $O
