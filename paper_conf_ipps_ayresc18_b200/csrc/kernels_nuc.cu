@@ -926,13 +926,19 @@ int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
   }
-  const int wops = std::min(nops, kMaxWin);
-  const size_t smem = S::bytes(wops);
-  int per_sm = 1;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G, W>, kThreads, smem);
-  const int resident = std::max(per_sm, 1) * nsm;
   const long long items = (long long)p * C;
   const int nchunks = (int)((items + kThreads - 1) / kThreads);
+  // a CTA walks the whole pass per chunk, so a second round of chunks doubles
+  // the pass: shrink the window until every chunk has its own resident CTA
+  int wops = std::min(nops, kMaxWin), per_sm = 1;
+  for (;;) {
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G, W>, kThreads,
+                                                  S::bytes(wops));
+    if ((long long)std::max(per_sm, 1) * nsm >= nchunks || wops <= 16) break;
+    wops = std::max(16, wops / 2);
+  }
+  const size_t smem = S::bytes(wops);
+  const int resident = std::max(per_sm, 1) * nsm;
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3((unsigned)std::min(nchunks, resident));
   cfg.blockDim = dim3(kThreads);
