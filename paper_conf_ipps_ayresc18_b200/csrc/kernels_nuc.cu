@@ -320,10 +320,11 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 // pattern of the children, and every operation maps item
 // (pattern, category) to the same thread here, so each thread's inputs in
 // level set k are its own outputs of earlier sets: program order replaces the
-// launch boundary, no grid or block synchronisation is needed.  Level sets
-// still bound the dependent chain: the G operations of a group (one set) issue
-// all their reads together, so a pass costs ~one memory round trip per set
-// (rerooting keeps its effect) instead of one launch per set.  A child made
+// launch boundary, no grid or block synchronisation is needed.  The G
+// operations of a group (one set) issue all their reads together.  Measured
+// (DESIGN.md §9 "Fused pass"): with ~8 warps per SM at configs[1] each warp's
+// serial walk over all operations is instruction-latency bound, so this is
+// slower than the per-set launches on a rerooted tree; opt-in only.  A child made
 // by one of the previous W-1 operations comes from the thread's own slot of a
 // shared-memory ring (host-resolved DevOp::ring1/ring2), so on a rerooted
 // pectinate tree the chain never leaves the SM.  Other reads of
