@@ -808,9 +808,17 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       I->h_ops[i] = d;
     }
     for (int k = 0; k < nsets; ++k) I->h_ops[offs[k + 1] - 1].flags |= OP_SET_END;
-    // fused pass: children produced by one of the previous W-1 ops are read
-    // from the thread's shared-memory ring (slot = producer index mod W)
+    // fused pass: a child produced by op j is read from the CTA's
+    // shared-memory ring (slot = j mod W) if no other op from the start of the
+    // producer's set to the end of the consumer's set -- the ops of one set run
+    // concurrently -- shares that slot: set_last(i) - set_first(j) < W
     const int W = fused_ring(I->prec);
+    std::vector<int> set_last(op_count), set_first(op_count);
+    for (int k = 0; k < nsets; ++k)
+      for (int i = offs[k]; i < offs[k + 1]; ++i) {
+        set_last[i] = offs[k + 1] - 1;
+        set_first[i] = offs[k];
+      }
     for (int i = 0; i < op_count; ++i) {
       DevOp &d = I->h_ops[i];
       int32_t *ring[2] = {&d.ring1, &d.ring2};
@@ -819,8 +827,9 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       for (int b = 0; b < 2; ++b) {
         *ring[b] = -1;
         if (d.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) continue;
-        for (int j = i - 1; j >= 0 && j > i - W; --j) {
+        for (int j = i - 1; j >= 0 && j > set_last[i] - W; --j) {
           if (ops[j].dest != ch[b]) continue;
+          if (set_last[i] - set_first[j] >= W) break;
           *ring[b] = j % W;
           if (cum[b] != nullptr && I->h_ops[j].scale_out == cum[b]) d.flags |= (b == 0 ? OP_RING_E1 : OP_RING_E2);
           break;

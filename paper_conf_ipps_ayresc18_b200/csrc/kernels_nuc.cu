@@ -340,25 +340,29 @@ template <typename T, int C, int W> struct FusedSmem {
   static size_t bytes(int wops) { return ring + (size_t)wops * per_op; }
 };
 
-template <typename T, int C, int G, int W>
-__global__ void __launch_bounds__(kThreads)
+template <typename T, int C, int G, int W, int H>
+__global__ void __launch_bounds__(kThreads * H)
 k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks, int wops) {
   using S = FusedSmem<T, C, W>;
   extern __shared__ __align__(16) unsigned char fsm[];
-  // per-thread ring of the last W operations' outputs (and cumulative
-  // exponents): a child produced by one of the previous W-1 ops is read back
-  // from shared memory, off the L2 round trip (DevOp::ring1/ring2)
+  // H groups of kThreads threads share the chunk's items: the ops of one
+  // level set are dealt round-robin (G at a time) to the groups, a barrier
+  // closes each set.  Ring of the last W operations' outputs (and cumulative
+  // exponents) per item: a child produced by a recent op is read back from
+  // shared memory, off the L2 round trip (DevOp::ring1/ring2, host-resolved so
+  // that no op running concurrently reuses the slot)
   T (*ringL)[kThreads][4] = reinterpret_cast<T (*)[kThreads][4]>(fsm);
   int (*ringE)[kThreads] = reinterpret_cast<int (*)[kThreads]>(fsm + (size_t)W * kThreads * 4 * sizeof(T));
   DevOp *sOps = reinterpret_cast<DevOp *>(fsm + S::ring);
   T *sP = reinterpret_cast<T *>(fsm + S::ring + (size_t)wops * sizeof(DevOp));
   uint8_t *sTip = reinterpret_cast<uint8_t *>(sP + (size_t)wops * 2 * C * 16);
-  const int cat = threadIdx.x % C;
-  const int lpat = threadIdx.x / C;
+  const int tid = threadIdx.x % kThreads, h = threadIdx.x / kThreads;
+  const int cat = tid % C;
+  const int lpat = tid / C;
   const unsigned nitems = (unsigned)p * C;
   pdl_wait();
   for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
-    const unsigned item = (unsigned)chunk * kThreads + threadIdx.x;
+    const unsigned item = (unsigned)chunk * kThreads + tid;
     const bool valid = item < nitems;
     const unsigned pat = valid ? item / C : 0u;
     for (int w0 = 0; w0 < nops; w0 += wops) {
@@ -369,18 +373,18 @@ k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks
       {
         const int4 *src = reinterpret_cast<const int4 *>(ops + w0);
         int4 *dst = reinterpret_cast<int4 *>(sOps);
-        for (int t = threadIdx.x; t < nw * (int)(sizeof(DevOp) / 16); t += kThreads) dst[t] = __ldg(src + t);
+        for (int t = threadIdx.x; t < nw * (int)(sizeof(DevOp) / 16); t += kThreads * H) dst[t] = __ldg(src + t);
       }
       __syncthreads();
       constexpr int kV = 16 / sizeof(T);              // elements per 16-byte vector
       constexpr int kPv = C * 16 / kV;                // vectors per branch
-      for (int t = threadIdx.x; t < nw * 2 * kPv; t += kThreads) {
+      for (int t = threadIdx.x; t < nw * 2 * kPv; t += kThreads * H) {
         const int o = t / (2 * kPv), r = t % (2 * kPv), br = r / kPv, v = r % kPv;
         const int4 *src = reinterpret_cast<const int4 *>(br == 0 ? sOps[o].P1 : sOps[o].P2);
         reinterpret_cast<int4 *>(sP)[t] = __ldg(src + v);
       }
       const unsigned pat0 = (unsigned)chunk * S::kPats;
-      for (int t = threadIdx.x; t < nw * 2 * S::kPats; t += kThreads) {
+      for (int t = threadIdx.x; t < nw * 2 * S::kPats; t += kThreads * H) {
         const int o = t / (2 * S::kPats), r = t % (2 * S::kPats), br = r / S::kPats, q = r % S::kPats;
         const DevOp &op = sOps[o];
         uint8_t code = 4u;
@@ -389,9 +393,13 @@ k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks
         sTip[t] = code;
       }
       __syncthreads();
-      for (int i = w0; i < w0 + nw;) {
-        int ng = 1;  // ops of this group: consecutive, within one level set and window
-        while (ng < G && i + ng < w0 + nw && !(sOps[i + ng - 1 - w0].flags & OP_SET_END)) ++ng;
+      for (int i0 = w0; i0 < w0 + nw;) {
+        int se = i0;  // this level set's ops within the window: [i0, se)
+        while (se < w0 + nw - 1 && !(sOps[se - w0].flags & OP_SET_END)) ++se;
+        ++se;
+        for (int base = i0; base < se; base += H * G) {
+        const int i = base + h * G;
+        const int ng = max(0, min(G, se - i));  // this group's ops (warp-uniform)
         T P1[G][16], P2[G][16], L1[G][4], L2[G][4];
         unsigned s1[G], s2[G];
         int ca[G], cb[G];
@@ -413,15 +421,15 @@ k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks
             for (int z = 0; z < 4; ++z) L1[j][z] = L2[j][z] = T(0);
             const int fl = op.flags, r1 = op.ring1, r2 = op.ring2;
             if (!(fl & OP_TIP1) && valid)
-              V4<T>::lds(r1 >= 0 ? &ringL[r1][threadIdx.x][0] : static_cast<const T *>(op.in1) + (size_t)item * 4,
+              V4<T>::lds(r1 >= 0 ? &ringL[r1][tid][0] : static_cast<const T *>(op.in1) + (size_t)item * 4,
                          L1[j]);
             if (!(fl & OP_TIP2) && valid)
-              V4<T>::lds(r2 >= 0 ? &ringL[r2][threadIdx.x][0] : static_cast<const T *>(op.in2) + (size_t)item * 4,
+              V4<T>::lds(r2 >= 0 ? &ringL[r2][tid][0] : static_cast<const T *>(op.in2) + (size_t)item * 4,
                          L2[j]);
             ca[j] = (sw && valid && cat == 0 && op.cum1 != nullptr)
-                        ? ((fl & OP_RING_E1) ? ringE[r1][threadIdx.x] : op.cum1[pat]) : 0;
+                        ? ((fl & OP_RING_E1) ? ringE[r1][tid] : op.cum1[pat]) : 0;
             cb[j] = (sw && valid && cat == 0 && op.cum2 != nullptr)
-                        ? ((fl & OP_RING_E2) ? ringE[r2][threadIdx.x] : op.cum2[pat]) : 0;
+                        ? ((fl & OP_RING_E2) ? ringE[r2][tid] : op.cum2[pat]) : 0;
           }
         }
 #pragma unroll
@@ -441,17 +449,19 @@ k_partials_nuc_fused(const DevOp *__restrict__ ops, int nops, int p, int nchunks
               const int e = frexp_exp(m);
               if (e != 0) scale_pow2(r, e);
               const int et = e + ca[j] + cb[j];
-              ringE[slot][threadIdx.x] = et;
+              ringE[slot][tid] = et;
               if (valid && cat == 0) op.scale_out[pat] = et;
             } else if (op.scale_in != nullptr) {
               const int e = valid ? op.scale_in[pat] : 0;
               if (e != 0) scale_pow2(r, e);
             }
-            V4<T>::st(&ringL[slot][threadIdx.x][0], r);
+            V4<T>::st(&ringL[slot][tid][0], r);
             if (valid) V4<T>::st(static_cast<T *>(op.out) + (size_t)item * 4, r);
           }
         }
-        i += ng;
+        }
+        if (H > 1) __syncthreads();  // the set's outputs are visible to every group
+        i0 = se;
       }
     }
   }
@@ -914,13 +924,14 @@ template <typename T, int C>
 int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   constexpr int G = 2;
   constexpr int W = fused_ring(sizeof(T) == 4 ? 32 : 64);
+  constexpr int H = 1;  // thread groups per CTA (H = 2 measured no faster)
   using S = FusedSmem<T, C, W>;
   constexpr size_t kBudget = 200 * 1024;
   constexpr int kMaxWin = (int)((kBudget - S::ring) / S::per_op);
   static_assert(kMaxWin >= 16, "fused window");
   static int nsm = 0;
   if (nsm == 0) {
-    cudaError_t e = cudaFuncSetAttribute(k_partials_nuc_fused<T, C, G, W>,
+    cudaError_t e = cudaFuncSetAttribute(k_partials_nuc_fused<T, C, G, W, H>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBudget);
     if (e != cudaSuccess) return (int)e;
     int dev = 0;
@@ -933,7 +944,7 @@ int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   // the pass: shrink the window until every chunk has its own resident CTA
   int wops = std::min(nops, kMaxWin), per_sm = 1;
   for (;;) {
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G, W>, kThreads,
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc_fused<T, C, G, W, H>, kThreads * H,
                                                   S::bytes(wops));
     if ((long long)std::max(per_sm, 1) * nsm >= nchunks || wops <= 16) break;
     wops = std::max(16, wops / 2);
@@ -942,7 +953,7 @@ int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   const int resident = std::max(per_sm, 1) * nsm;
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3((unsigned)std::min(nchunks, resident));
-  cfg.blockDim = dim3(kThreads);
+  cfg.blockDim = dim3(kThreads * H);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute at[1];
@@ -950,7 +961,7 @@ int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_fused<T, C, G, W>, d_ops, nops, p, nchunks, wops);
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_nuc_fused<T, C, G, W, H>, d_ops, nops, p, nchunks, wops);
 }
 
 template <typename T>
