@@ -177,9 +177,20 @@ int rrl_set_tip_partials(int inst, int tip, const double *partials /*[p][s]*/);
 /* Arbitrary partials for any buffer (tests / restarts), layout [c][p][s]. */
 int rrl_set_partials(int inst, int buffer, const double *partials);
 int rrl_get_partials(int inst, int buffer, double *out /*[c][p][s]*/);
+/* Pattern weights wt_i: the multiplicity of unique site pattern i (PAPER.md:169
+ * "--sites ... site patterns", :180 "unique site patterns"; reading A15),
+ * applied only in the root/edge sum lnL = sum_i wt_i lnL_i.  Default 1. */
 int rrl_set_pattern_weights(int inst, const double *w /*[p]*/);
+/* Stationary frequencies pi of model slot idx: the root distribution of the
+ * root/edge integration (reading A4; Felsenstein [7]).  Reroot
+ * invariance holds only for the stationary pi of a reversible
+ * model.  Default uniform. */
 int rrl_set_state_frequencies(int inst, int idx, const double *pi /*[s]*/);
+/* Rate multipliers r_c of the +Gamma categories (reading A3: P_c =
+ * exp(Q r_c t), categories combined only at the root), every model slot. */
 int rrl_set_category_rates(int inst, const double *r /*[c]*/);
+/* Category weights w_c of model slot idx for the root/edge integration
+ * (reading A3/A4).  Default 1/c. */
 int rrl_set_category_weights(int inst, int idx, const double *w /*[c]*/);
 /* Category rates of model slot idx (0 <= idx < eigen_count) for partitioned
  * analyses ("independent model parameters for each of these
@@ -259,9 +270,14 @@ int rrl_calculate_edge_log_likelihoods(int inst, int parent_buffer, int child_bu
                                        int matrix_idx, int cat_weights_idx, int freqs_idx,
                                        int parent_scale_idx, int child_scale_idx,
                                        double *out_sum);
+/* Per-pattern lnL_i of the last root/edge call (reading A4; each
+ * pattern's likelihood is computed autonomously and combined afterwards). */
 int rrl_get_site_log_likelihoods(int inst, double *out /*[p]*/);
 
-/* ------------------------------------------------------------- profiling */
+/* ------------------------------------------------------------- profiling
+ * The paper's metric is the throughput of the partial-likelihood kernel only
+ * (§VI-C, --full-timing PAPER.md:180): these counters time
+ * the updatePartials launches separately from K1/K4/K5 (reading A17). */
 int rrl_set_profiling(int inst, int enable);
 int rrl_get_profile(int inst, rrl_profile *out); /* synchronizes the stream */
 int rrl_reset_profile(int inst);
@@ -322,6 +338,60 @@ int rrl_schedule_partial(int tip_count, const int32_t *parent, const int32_t *no
  * cost comparisons.  blen may be NULL. */
 int rrl_reroot_exhaustive(int tip_count, const int32_t *parent, const double *blen,
                           int32_t *out_root_edge, int32_t *out_set_count);
+
+/* Topology moves (host; SURVEY.md NEXT-2, §VII-D "only a subtree
+ * representing the modified portion of the overall tree is recomputed for
+ * each topology change").  Node ids and the root id are kept; the input tree
+ * is not modified; out_parent[2n-1] / out_blen[2n-1] receive the new tree.
+ * SPR (reading A26): prune the subtree at prune_node (a non-root node whose
+ *   parent p is not the root): p's other child s takes p's place, branch
+ *   t_s + t_p; regraft p on the branch above regraft_node (not the root, not
+ *   p, not inside the pruned subtree), splitting it in halves.
+ *   RRL_ERROR_OUT_OF_RANGE for an illegal pair.
+ * NNI (reading A27) on the unrooted internal edge keyed by edge_node (the
+ *   branch above it; the root's merged branch is keyed by the root's smaller
+ *   child, which must then be internal, as must the other root child):
+ *   edge_node's child `which` (0 = smaller id) and the subtree across the
+ *   edge (the sibling, or the other root child's smaller child) exchange
+ *   places, keeping their branch lengths. */
+int rrl_tree_spr(int tip_count, const int32_t *parent, const double *blen, int prune_node,
+                 int regraft_node, int32_t *out_parent, double *out_blen);
+int rrl_tree_nni(int tip_count, const int32_t *parent, const double *blen, int edge_node, int which,
+                 int32_t *out_parent, double *out_blen);
+
+/* Partial update after any change (SURVEY.md NEXT-2; PAPER.md:258, :268,
+ * :282-288; reading A28).  The partials buffers (identity assignment: buffer
+ * = node id) hold the partials of the stored tree (stored_parent /
+ * stored_blen).  For the new tree (parent / blen, same tip set), a node's
+ * stored partial is reused iff its children, their branch lengths and,
+ * recursively, their subtrees are unchanged; every other internal node is
+ * recomputed.  flags = RRL_SCHED_LEVEL: on the new tree's rooting.
+ * flags = RRL_SCHED_REROOT: on the rooting (over all 2n-3 edges, O(n)) that
+ * minimises the number of sets of this update, then the number of
+ * operations (rerooting also recomputes every node whose orientation flips),
+ * then keeps the current root edge, then the smallest key; the rerooted tree
+ * is built as by rrl_reroot_and_schedule.
+ * Outputs: out_parent / out_blen (the tree the ops refer to; use its branch
+ * lengths for the transition matrices), out_root_edge, out_ops[<= n-1] (same
+ * conventions as rrl_reroot_and_schedule, identity buffers), out_set_offsets
+ * [<= n], out_op_count, out_set_count.  Any output may be NULL. */
+int rrl_schedule_update(int tip_count, const int32_t *stored_parent, const double *stored_blen,
+                        const int32_t *parent, const double *blen, uint32_t flags, int32_t *out_parent,
+                        double *out_blen, int32_t *out_root_edge, rrl_op *out_ops,
+                        int32_t *out_set_offsets, int32_t *out_op_count, int32_t *out_set_count);
+
+/* Predicted time (microseconds) of one updatePartials pass over `ops` /
+ * `set_offsets` (SURVEY.md NEXT-4; PAPER.md:270, :288 cost vs benefit of
+ * rerooting): sum over level sets k of
+ *   launch_us + (B_k - phi_k C_k) / hbm_gbs,
+ * B_k = the set's algorithmic bytes (per pattern: every output c s B + 4,
+ * every internal child c s B + 4, every tip child 1), C_k = its reads of
+ * children written by set k-1, phi_k = clamp(1 - O_{k-1} / l2_bytes, 0, 1)
+ * with O_{k-1} = set k-1's output bytes (the part still in L2).  B = precision
+ * / 8.  Used to decide whether rerooting pays (DESIGN.md §9 "NEXT-4"). */
+int rrl_schedule_cost(int tip_count, const rrl_op *ops, int op_count, const int32_t *set_offsets,
+                      int set_count, int pattern_count, int state_count, int category_count, int precision,
+                      double launch_us, double hbm_gbs, double l2_bytes, double *out_us);
 
 /* Substitution model (host, fp64): builds the normalised rate matrix Q
  * (-sum_i pi_i Q_ii = 1) for model in {"jc69","hky","gtr","gy94"} and its

@@ -727,6 +727,14 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
   if (!same) {
     // --- validate
     std::vector<int> stamp(I->n_buf, -1);
+    // per-node (non-cumulative) exponents are only summed after the call (K5),
+    // so two ops of one call writing the same scale buffer would lose the first
+    // op's exponents: rejected (recycled buffers need RRL_FLAG_SCALE_CUMULATIVE)
+    std::vector<int> scale_writer(cumulative ? 0 : I->n_scale, -1);
+    // ranged calls: ops of one set writing the same buffer must cover disjoint
+    // pattern ranges (different partitions of one node)
+    std::vector<std::vector<std::pair<int, int>>> dest_ranges;
+    if (ranges) dest_ranges.resize(I->n_buf);
     for (int k = 0; k < nsets; ++k) {
       for (int i = offs[k]; i < offs[k + 1]; ++i) {
         const rrl_op &o = ops[i];
@@ -742,7 +750,25 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
           if (ch < I->n_tips && !I->has_states[ch] && !I->tip_partials[ch])
             return fail(RRL_ERROR_GENERAL, "tip without data");
         if (stamp[o.dest] == k && !ranges) return fail(RRL_ERROR_GENERAL, "two ops write one buffer in a set");
+        if (ranges) {
+          auto &dr = dest_ranges[o.dest];
+          if (stamp[o.dest] != k) dr.clear();
+          const int b = ranges[2 * i], e = ranges[2 * i + 1];
+          for (const auto &q : dr)
+            if (b < q.second && q.first < e)
+              return fail(RRL_ERROR_GENERAL, "two ops of a set write overlapping pattern ranges of one buffer");
+          dr.push_back({b, e});
+        }
         stamp[o.dest] = k;
+        if (!cumulative && o.dest_scale_write >= 0) {
+          const int prev = scale_writer[o.dest_scale_write];
+          // (partition copies of one node: same dest in the same set, ranges checked disjoint above)
+          if (prev >= 0 && !(ranges && ops[prev].dest == o.dest && prev >= offs[k]))
+            return fail(RRL_ERROR_GENERAL,
+                        "two ops write one scale buffer in one call (per-node exponents would be lost "
+                        "before accumulation; use distinct scale buffers or RRL_FLAG_SCALE_CUMULATIVE)");
+          scale_writer[o.dest_scale_write] = i;
+        }
         if (cumulative && o.dest_scale_write >= 0) {
           if (o.dest_scale_write != o.dest - I->n_tips)
             return fail(RRL_ERROR_GENERAL, "cumulative scaling needs dest_scale_write = dest - tip_count");
@@ -812,15 +838,20 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
     // shared-memory ring (slot = j mod W) if no other op from the start of the
     // producer's set to the end of the consumer's set -- the ops of one set run
     // concurrently -- shares that slot: set_last(i) - set_first(j) < W
+    const bool fused_desc = I->s == 4 && (I->flags & RRL_FLAG_FUSED_PASS) && !ranges;
     const int W = fused_ring(I->prec);
-    std::vector<int> set_last(op_count), set_first(op_count);
-    for (int k = 0; k < nsets; ++k)
+    std::vector<int> set_last(fused_desc ? op_count : 0), set_first(fused_desc ? op_count : 0);
+    for (int k = 0; k < nsets && fused_desc; ++k)
       for (int i = offs[k]; i < offs[k + 1]; ++i) {
         set_last[i] = offs[k + 1] - 1;
         set_first[i] = offs[k];
       }
     for (int i = 0; i < op_count; ++i) {
       DevOp &d = I->h_ops[i];
+      if (!fused_desc) {  // ring slots are read only by the fused-pass kernel
+        d.ring1 = d.ring2 = -1;
+        continue;
+      }
       int32_t *ring[2] = {&d.ring1, &d.ring2};
       const int ch[2] = {ops[i].child1, ops[i].child2};
       const int32_t *cum[2] = {d.cum1, d.cum2};

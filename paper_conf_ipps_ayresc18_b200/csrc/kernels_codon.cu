@@ -238,7 +238,8 @@ k_partials_codon(const DevOp *__restrict__ ops, int p, int p_pad) {
 template <typename T, int C>
 int launch_codon_t(const DevOp *d_ops, int nops, int p, int p_pad, cudaStream_t st) {
   const size_t smem = sizeof(CodonSmem<T>);
-  static bool configured = false;
+  static bool configured_dev[kMaxDevices] = {};
+  bool &configured = configured_dev[device_slot()];
   if (!configured) {
     cudaError_t e = cudaFuncSetAttribute(k_partials_codon<T, C>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);

@@ -485,7 +485,8 @@ k_partials_codon_tc(const DevOp *__restrict__ ops, int p, int p_pad, int ntiles,
 
 template <int C>
 int launch_tc(const DevOp *d_ops, int nops, int p, int p_pad, cudaStream_t st) {
-  static int nsm = 0;
+  static int nsm_dev[kMaxDevices] = {};
+  int &nsm = nsm_dev[device_slot()];
   if (nsm == 0) {
     cudaError_t e = cudaFuncSetAttribute(k_partials_codon_tc<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          SMEM_TOTAL);

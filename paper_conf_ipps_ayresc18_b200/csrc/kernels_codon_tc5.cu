@@ -542,7 +542,8 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
 template <int C>
 int launch_tc5(const DevOp *d_ops, int nops, int p, int p_pad, const CUtensorMap *tA, const CUtensorMap *tP,
                const CUtensorMap *tPlo, cudaStream_t st) {
-  static int nsm = 0;
+  static int nsm_dev[kMaxDevices] = {};
+  int &nsm = nsm_dev[device_slot()];
   if (nsm == 0) {
     cudaError_t e = cudaFuncSetAttribute(k_partials_codon_tc5<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          SMEM_TOTAL);

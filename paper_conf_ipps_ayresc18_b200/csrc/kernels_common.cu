@@ -7,6 +7,12 @@
 #include "rrl_internal.h"
 
 namespace rrl {
+
+int device_slot() {
+  int d = 0;
+  cudaGetDevice(&d);
+  return d < 0 ? 0 : (d < kMaxDevices ? d : kMaxDevices - 1);
+}
 namespace {
 
 constexpr double kLn2 = 0.693147180559945309417232121458176568;
@@ -290,7 +296,8 @@ int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *
   if (s_pad == 64) {  // codon: register-tiled, persistent blocks over (matrix, category) items
     const size_t smem64 = sizeof(double) * (2 * 64 * 64 + 64);
     const int items = count * c;
-    static int grid_cap = 0;
+    static int grid_caps[kMaxDevices] = {};
+    int &grid_cap = grid_caps[device_slot()];
     if (grid_cap == 0) {
       int dev = 0, nsm = 0, per = 0;
       cudaGetDevice(&dev);

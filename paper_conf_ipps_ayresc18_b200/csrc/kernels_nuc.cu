@@ -851,8 +851,9 @@ int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, in
 // trip, so the widest single round wins.
 template <typename T, int C>
 int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int early, cudaStream_t st) {
-  static int resident = -1;  // per template instance
-  if (resident < 0) {
+  static int resident_dev[kMaxDevices] = {};  // per template instance and device
+  int &resident = resident_dev[device_slot()];
+  if (resident <= 0) {
     int per_sm = 1, dev = 0, nsm = 148;
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, 1>, kThreads, 0);
     cudaGetDevice(&dev);
@@ -869,9 +870,11 @@ int launch_bulk(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   const long long total = (long long)nops * nchunks;
   if (total > 0x7fffffffLL) return (int)cudaErrorInvalidValue;
   const size_t smem = sizeof(BulkStage<T, C>) * kStages;
-  static int per_sm = -1;  // per template instance
-  static int nsm = 0;
-  if (per_sm < 0) {
+  static int per_sm_dev[kMaxDevices] = {};  // per template instance and device
+  static int nsm_dev[kMaxDevices] = {};
+  const int slot = device_slot();
+  int &per_sm = per_sm_dev[slot], &nsm = nsm_dev[slot];
+  if (per_sm <= 0) {
     cudaError_t e = cudaFuncSetAttribute(k_partials_nuc_bulk<T, C, kStages>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return (int)e;
@@ -929,7 +932,8 @@ int launch_fused_t(const DevOp *d_ops, int nops, int p, cudaStream_t st) {
   constexpr size_t kBudget = 200 * 1024;
   constexpr int kMaxWin = (int)((kBudget - S::ring) / S::per_op);
   static_assert(kMaxWin >= 16, "fused window");
-  static int nsm = 0;
+  static int nsm_dev[kMaxDevices] = {};
+  int &nsm = nsm_dev[device_slot()];
   if (nsm == 0) {
     cudaError_t e = cudaFuncSetAttribute(k_partials_nuc_fused<T, C, G, W, H>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBudget);

@@ -11,6 +11,13 @@ namespace rrl {
 // Records a thread-local error message and returns `code`.
 int fail(int code, const std::string &msg);
 
+// Kernel attributes (dynamic shared-memory opt-in) and SM counts are per
+// device context: launchers cache them per device slot (the current device,
+// clamped to kMaxDevices - 1), so instances on different GPUs of one process
+// each configure their own device.
+constexpr int kMaxDevices = 64;
+int device_slot();
+
 // Resolved operation descriptor, one per rrl_op, resident in device memory.
 // The multi-operation kernel reads its descriptor by blockIdx.y ("pointer
 // arithmetic to allow different input and output arrays for different

@@ -366,3 +366,241 @@ extern "C" int rrl_reroot_exhaustive(int tip_count, const int32_t *parent, const
     return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_reroot_exhaustive");
   }
 }
+
+// ---------------------------------------------------------------------------
+// Topology moves (§VII-D "only a subtree
+// representing the modified portion of the overall tree is recomputed for each
+// topology change").  The paper does not define the moves: DESIGN.md readings
+// A26 (SPR) and A27 (NNI).  Node ids and the root are kept.
+extern "C" int rrl_tree_spr(int tip_count, const int32_t *parent, const double *blen, int prune_node,
+                            int regraft_node, int32_t *out_parent, double *out_blen) {
+  try {
+    if (!blen || !out_parent || !out_blen) return rrl::fail(RRL_ERROR_GENERAL, "NULL array");
+    View v;
+    int rc = build_view(tip_count, parent, v);
+    if (rc < 0) return rc;
+    const int N = v.N, R = v.root, x = prune_node, r = regraft_node;
+    if (x < 0 || x >= N || x == R) return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "prune node must be a non-root node");
+    const int p = v.parent[x];
+    if (p == R) return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "prune node's parent must not be the root");
+    if (r < 0 || r >= N || r == R || r == p) return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "bad regraft node");
+    for (int y = r; y != -1; y = v.parent[y])
+      if (y == x) return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "regraft node inside the pruned subtree");
+    std::vector<int32_t> par(v.parent.begin(), v.parent.end());
+    std::vector<double> bl(blen, blen + N);
+    const int g = v.parent[p];
+    const int s = (v.c1[p] == x) ? v.c2[p] : v.c1[p];
+    par[s] = g;  // prune: the sibling takes p's place, branches merge
+    bl[s] = bl[s] + bl[p];
+    const int q = par[r];  // regraft: p on the branch above r, split in halves
+    const double half = bl[r] / 2.0;
+    par[p] = q;
+    bl[p] = half;
+    par[r] = p;
+    bl[r] = half;
+    std::copy(par.begin(), par.end(), out_parent);
+    std::copy(bl.begin(), bl.end(), out_blen);
+    return RRL_SUCCESS;
+  } catch (...) {
+    return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_tree_spr");
+  }
+}
+
+extern "C" int rrl_tree_nni(int tip_count, const int32_t *parent, const double *blen, int edge_node, int which,
+                            int32_t *out_parent, double *out_blen) {
+  try {
+    if (!blen || !out_parent || !out_blen) return rrl::fail(RRL_ERROR_GENERAL, "NULL array");
+    View v;
+    int rc = build_view(tip_count, parent, v);
+    if (rc < 0) return rc;
+    const int n = v.n, N = v.N, R = v.root, x = edge_node;
+    if (x < n || x >= N || x == R || (which != 0 && which != 1))
+      return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "NNI needs an internal non-root node and which in {0, 1}");
+    std::vector<int32_t> par(v.parent.begin(), v.parent.end());
+    const int u = v.parent[x];
+    const int mine = which == 0 ? v.c1[x] : v.c2[x];
+    if (u == R) {
+      const int a = v.c1[R], b = v.c2[R];
+      if (x != a) return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "the root's merged edge is keyed by its smaller child");
+      if (b < n) return rrl::fail(RRL_ERROR_OUT_OF_RANGE, "merged root edge is not internal");
+      const int theirs = v.c1[b];
+      par[mine] = b;
+      par[theirs] = x;
+    } else {
+      const int w = (v.c1[u] == x) ? v.c2[u] : v.c1[u];
+      par[mine] = u;
+      par[w] = x;
+    }
+    std::copy(par.begin(), par.end(), out_parent);
+    std::copy(blen, blen + N, out_blen);
+    return RRL_SUCCESS;
+  } catch (...) {
+    return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_tree_nni");
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Partial update after any change (moves, branch lengths), optionally
+// rerooted (reading A28).
+// A node's stored partial (identity buffers) is reused iff its children, their
+// branch lengths and, recursively, their subtrees equal the stored tree's: one
+// O(n) pass.  Rerooting on the edge above x flips every node strictly between
+// x and the root (x_1..x_k: their children change) and the root itself; all
+// other nodes keep their rooted subtree.  So for every candidate edge the
+// update's set count is 1 + max(dirty height below x, dirty height of the
+// flipped side), computed for all 2n-3 edges by the same down/up passes as the
+// full reroot (edge_table), with the flipped side always recomputed, and its
+// operation count is |D| + (valid nodes among x_1..x_k) + (root valid).
+extern "C" int rrl_schedule_update(int tip_count, const int32_t *stored_parent, const double *stored_blen,
+                                   const int32_t *parent, const double *blen, uint32_t flags,
+                                   int32_t *out_parent, double *out_blen, int32_t *out_root_edge,
+                                   rrl_op *out_ops, int32_t *out_set_offsets, int32_t *out_op_count,
+                                   int32_t *out_set_count) {
+  try {
+    if (!stored_blen || !blen) return rrl::fail(RRL_ERROR_GENERAL, "blen is NULL");
+    const uint32_t mode = flags & 0xffu;
+    if (mode != RRL_SCHED_LEVEL && mode != RRL_SCHED_REROOT)
+      return rrl::fail(RRL_ERROR_GENERAL, "rrl_schedule_update: mode must be LEVEL or REROOT");
+    View s, v;
+    int rc = build_view(tip_count, stored_parent, s);
+    if (rc < 0) return rc;
+    rc = build_view(tip_count, parent, v);
+    if (rc < 0) return rc;
+    const int n = v.n, N = v.N, R = v.root, a = v.c1[R], b = v.c2[R];
+    std::vector<char> valid(N, 1);
+    std::vector<int> down(N, 0);
+    int ndirty = 0;
+    for (int x : v.post) {
+      const int l = v.c1[x], r = v.c2[x];
+      valid[x] = (s.c1[x] == l && s.c2[x] == r && stored_blen[l] == blen[l] && stored_blen[r] == blen[r] &&
+                  valid[l] && valid[r]);
+      if (!valid[x]) {
+        down[x] = 1 + std::max(down[l], down[r]);
+        ++ndirty;
+      }
+    }
+    const int cur = std::min(a, b);
+    int key = cur, best_sets = down[R];
+    if (mode == RRL_SCHED_REROOT && ndirty > 0) {
+      std::vector<int> up(N, 0), cnt(N, 0);
+      up[a] = down[b];
+      up[b] = down[a];
+      for (auto it = v.post.rbegin(); it != v.post.rend(); ++it) {  // parents first
+        const int u = *it;
+        if (u == R) continue;
+        const int l = v.c1[u], r = v.c2[u];
+        up[l] = 1 + std::max(down[r], up[u]);
+        up[r] = 1 + std::max(down[l], up[u]);
+        cnt[l] = cnt[r] = cnt[u] + (valid[u] ? 1 : 0);
+      }
+      // (sets, ops, not current, key), reading A28
+      long long best[4] = {down[R], ndirty, 0, cur};
+      for (int x = 0; x < N; ++x) {
+        if (x == R || x == a || x == b) continue;
+        const long long row[4] = {1 + std::max(down[x], up[x]), ndirty + cnt[x] + (valid[R] ? 1 : 0), 1, x};
+        if (std::lexicographical_compare(row, row + 4, best, best + 4)) std::copy(row, row + 4, best);
+      }
+      key = (int)best[3];
+      best_sets = (int)best[0];
+    }
+    std::vector<int> par;
+    std::vector<double> bl;
+    reroot(v, blen, key, par, bl);
+    View w;
+    rc = build_view(n, par.data(), w);
+    if (rc < 0) return rc;
+    std::vector<char> dirty(N, 0);
+    for (int x = n; x < N; ++x) dirty[x] = !valid[x];
+    if (key != cur) {
+      dirty[R] = 1;
+      for (int y = v.parent[key]; y != R; y = v.parent[y]) dirty[y] = 1;
+    }
+    std::vector<int> lev(N, 0);
+    int H = 0, cnt_ops = 0;
+    for (int x : w.post)
+      if (dirty[x]) {
+        lev[x] = 1 + std::max(dirty[w.c1[x]] ? lev[w.c1[x]] : 0, dirty[w.c2[x]] ? lev[w.c2[x]] : 0);
+        H = std::max(H, lev[x]);
+        ++cnt_ops;
+      }
+    if (H != best_sets) return rrl::fail(RRL_ERROR_GENERAL, "internal: update set count mismatch");
+    std::vector<int> count(H + 2, 0), offs(H + 1, 0);
+    for (int x = n; x < N; ++x)
+      if (dirty[x]) ++count[lev[x]];
+    for (int k = 1; k <= H; ++k) offs[k] = offs[k - 1] + count[k];
+    std::vector<int> fill(offs.begin(), offs.end()), order(cnt_ops);
+    for (int x = n; x < N; ++x)
+      if (dirty[x]) order[fill[lev[x] - 1]++] = x;
+    if (out_parent) std::copy(par.begin(), par.end(), out_parent);
+    if (out_blen) std::copy(bl.begin(), bl.end(), out_blen);
+    if (out_root_edge) *out_root_edge = key;
+    if (out_ops)
+      for (int i = 0; i < cnt_ops; ++i) {
+        const int x = order[i];
+        out_ops[i] = rrl_op{x, x - n, RRL_NONE, w.c1[x], w.c1[x], w.c2[x], w.c2[x]};
+      }
+    if (out_set_offsets) std::copy(offs.begin(), offs.end(), out_set_offsets);
+    if (out_op_count) *out_op_count = cnt_ops;
+    if (out_set_count) *out_set_count = H;
+    return RRL_SUCCESS;
+  } catch (...) {
+    return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_schedule_update");
+  }
+}
+
+// ---------------------------------------------------------------------------
+// Schedule cost model ("the desired
+// outcome is that the benefit gained by the increased concurrent computation
+// on the rerooted tree is greater than the cost").  Per level set k:
+//   T_k = t0 + (B_k - phi_k C_k) / BW,
+// B_k = algorithmic bytes of the set (every op: output c s B + 4 B exponent;
+// each internal child c s B + 4 B cumulative exponent, each tip child 1 B, per
+// pattern), C_k = the part of it that reads children written by set k-1, and
+// phi_k = clamp(1 - O_{k-1} / L2, 0, 1) the fraction of set k-1's output
+// O_{k-1} still in L2.  t0 is the fixed cost of a level-set launch.  Fitted
+// against the measured 1,024-pectinate sweep (DESIGN.md §9 "NEXT-4"): it
+// predicts rerooting to win up to ~10^5 patterns and to lose at 10^6 (fp32),
+// where a one-op chain re-reads its child from L2.
+extern "C" int rrl_schedule_cost(int tip_count, const rrl_op *ops, int op_count, const int32_t *set_offsets,
+                                 int set_count, int pattern_count, int state_count, int category_count,
+                                 int precision, double launch_us, double hbm_gbs, double l2_bytes,
+                                 double *out_us) {
+  try {
+    if (!ops || !set_offsets || !out_us || set_count < 0 || op_count < 0 || tip_count < 2 || pattern_count < 0 ||
+        (precision != 32 && precision != 64) || hbm_gbs <= 0.0 || l2_bytes < 0.0)
+      return rrl::fail(RRL_ERROR_GENERAL, "rrl_schedule_cost: bad arguments");
+    if (set_offsets[0] != 0 || set_offsets[set_count] != op_count)
+      return rrl::fail(RRL_ERROR_GENERAL, "rrl_schedule_cost: set offsets must span ops");
+    const double p = pattern_count;
+    const double vec = (double)category_count * state_count * (precision / 8);
+    const double out_b = (vec + 4.0) * p, int_b = (vec + 4.0) * p, tip_b = 1.0 * p;
+    int maxbuf = tip_count;
+    for (int i = 0; i < op_count; ++i) maxbuf = std::max({maxbuf, ops[i].dest + 1, ops[i].child1 + 1, ops[i].child2 + 1});
+    std::vector<int> written_in(maxbuf, -2);
+    double total = 0.0, prev_out = 0.0;
+    for (int k = 0; k < set_count; ++k) {
+      double B = 0.0, Cprev = 0.0, O = 0.0;
+      for (int i = set_offsets[k]; i < set_offsets[k + 1]; ++i) {
+        const rrl_op &o = ops[i];
+        for (int ch : {o.child1, o.child2}) {
+          if (ch < tip_count) {
+            B += tip_b;
+          } else {
+            B += int_b;
+            if (written_in[ch] == k - 1) Cprev += int_b;
+          }
+        }
+        B += out_b;
+        O += out_b;
+      }
+      const double phi = l2_bytes > 0.0 ? std::min(1.0, std::max(0.0, 1.0 - prev_out / l2_bytes)) : 0.0;
+      total += launch_us + (B - phi * Cprev) / (hbm_gbs * 1e3);  // bytes / (GB/s) -> us
+      for (int i = set_offsets[k]; i < set_offsets[k + 1]; ++i) written_in[ops[i].dest] = k;
+      prev_out = O;
+    }
+    *out_us = total;
+    return RRL_SUCCESS;
+  } catch (...) {
+    return rrl::fail(RRL_ERROR_UNIDENTIFIED_EXCEPTION, "exception in rrl_schedule_cost");
+  }
+}

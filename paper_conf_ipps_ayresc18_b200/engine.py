@@ -89,12 +89,36 @@ class TreeLikelihood:
         self.ranges = [(int(b), int(e)) for b, e in ranges]
 
     def set_tips(self, tips_u8: np.ndarray):
-        R.rrl_set_tip_states_u8(self.inst, 0, tips_u8)
+        R.rrl_set_tip_states_u8(self.inst, 0, tips_u8, self.p)
 
     def set_pattern_weights(self, w):
         R.rrl_set_pattern_weights(self.inst, w)
 
+    # NEXT-4 cost model parameters (rrl_schedule_cost): fixed cost of one
+    # level-set launch and sustained HBM bandwidth, fitted to the measured
+    # 1,024-pectinate sweep (DESIGN.md §9 "NEXT-4"); L2 size of the device.
+    launch_us = 2.0
+    hbm_gbs = 6225.0
+    l2_bytes = 126e6
+
+    def predicted_us(self, sch) -> float:
+        return R.rrl_schedule_cost(self.n, sch["ops"], sch["set_offsets"], self.p, self.s, self.c,
+                                   self.precision, self.launch_us, self.hbm_gbs, self.l2_bytes)
+
     def set_tree(self, parent, blen, mode: str = "reroot", reuse_buffers: bool = False):
+        """mode: "sequential" | "level" | "reroot" | "auto" -- auto reroots only
+        when the cost model predicts the rerooted schedule to be faster
+        (NEXT-4; PAPER.md:270, :288)."""
+        if reuse_buffers and not self.cumulative:
+            # recycled buffers recycle their scale buffers too: per-node exponents
+            # of consumed children would be overwritten before K5 sums them
+            raise ValueError("reuse_buffers needs cumulative_scaling=True")
+        if mode == "auto":
+            cand = [R.rrl_reroot_and_schedule(self.n, parent, blen, m, reuse_buffers) for m in ("reroot", "level")]
+            cost = [self.predicted_us(c) for c in cand]
+            self.auto_choice = {"reroot_us": cost[0], "level_us": cost[1],
+                                "mode": "reroot" if cost[0] <= cost[1] else "level"}
+            mode = self.auto_choice["mode"]
         sch = R.rrl_reroot_and_schedule(self.n, parent, blen, mode, reuse_buffers)
         if sch["buffer_count"] > self.nbuf:
             raise ValueError(f"schedule needs {sch['buffer_count']} buffers, instance has {self.nbuf}")
@@ -106,11 +130,43 @@ class TreeLikelihood:
         ops = sch["ops"]
         # physical buffer holding the root (last op of the last set)
         self.root_buffer = int(ops["dest"][-1])
-        if not self.cumulative:
-            ops = ops.copy()
         self.sched = sch
+        self.reuse = reuse_buffers
+        self.tree_parent, self.tree_blen = par.copy(), sch["blen"].copy()
         self.ops = ops
         self.offsets = sch["set_offsets"]
+        self._pops = None
+        return sch
+
+    def update_tree(self, parent, blen, reroot: bool = False) -> dict:
+        """Bring the stored partials up to date for a changed tree (topology
+        moves, branch lengths; NEXT-2): only the nodes whose
+        rooted subtree changed are recomputed (rrl_schedule_update, reading
+        A28), level-batched, optionally on the rooting that minimises this
+        update's sets.  K1 refreshes every matrix (one launch).  Needs identity
+        buffers and a previous full pass.  Returns the update schedule."""
+        if self.sched is None or self.reuse or self.partitions > 1:
+            raise ValueError("update_tree needs a full pass on identity buffers first")
+        sch = R.rrl_schedule_update(self.n, self.tree_parent, self.tree_blen, parent, blen, reroot)
+        par = sch["parent"]
+        nonroot = np.flatnonzero(par >= 0).astype(np.int32)
+        self.matrix_idx = nonroot
+        self.t = sch["blen"][nonroot].copy()
+        R.rrl_update_transition_matrices(self.inst, 0, self.matrix_idx, self.t)
+        if sch["op_count"] > 0:
+            R.rrl_update_partials(self.inst, sch["ops"], sch["set_offsets"])
+        if not self.cumulative:  # per-node exponents: re-sum every internal node's
+            cum = self.n_scale - 1
+            R.rrl_reset_scale_factors(self.inst, cum)
+            R.rrl_accumulate_scale_factors(self.inst, np.arange(self.n - 1, dtype=np.int32), cum)
+        self.root = int(np.flatnonzero(par < 0)[0])
+        self.root_buffer = self.root
+        self.tree_parent, self.tree_blen = par.copy(), sch["blen"].copy()
+        # later full passes run the level sets of the tree as it now stands
+        full = R.rrl_reroot_and_schedule(self.n, par, sch["blen"], "level")
+        self.sched = full
+        self.ops = full["ops"]
+        self.offsets = full["set_offsets"]
         self._pops = None
         return sch
 

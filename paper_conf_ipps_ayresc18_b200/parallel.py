@@ -37,9 +37,15 @@ def schedule_digest(sched: dict) -> str:
 
 
 def allreduce_sum_(tensor, group=None):
-    """In-place SUM all-reduce of a 1-element fp64 tensor (device tensor with
-    NCCL; CPU tensor with gloo)."""
+    """In-place SUM all-reduce of a 1-element fp64 tensor: on the device with
+    NCCL; through a host copy with gloo (the CPU-side wiring tests and
+    several ranks sharing one GPU, where NCCL refuses)."""
     import torch.distributed as dist
+    if tensor.is_cuda and dist.get_backend(group) != "nccl":
+        h = tensor.cpu()
+        dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
+        tensor.copy_(h)
+        return tensor
     dist.all_reduce(tensor, op=dist.ReduceOp.SUM, group=group)
     return tensor
 
@@ -57,8 +63,14 @@ class ShardedTreeLikelihood:
         if self.hi <= self.lo:
             raise ValueError("empty pattern slice: use fewer ranks than patterns")
         self.group = group
+        if stream_ptr is None:
+            # the collective runs on torch's current stream: the library must
+            # enqueue K4 on that same stream so all_reduce is ordered after it
+            stream_ptr = torch.cuda.current_stream(device).cuda_stream
         self.tl = TreeLikelihood(n, self.hi - self.lo, s, c, precision=precision, device=device,
                                  cuda_graph=cuda_graph, stream_ptr=stream_ptr)
+        self.stream_ptr = stream_ptr
+        self.device = device
         self.d_out = torch.zeros(1, dtype=torch.float64, device=f"cuda:{device}")
 
     def set_model_params(self, mp, rates, cat_weights):
@@ -77,6 +89,12 @@ class ShardedTreeLikelihood:
         """Local pass + in-place all-reduce; returns the device tensor."""
         self.tl.update()
         self.tl.root_loglik_device(self.d_out.data_ptr())
+        import torch
+        if torch.cuda.current_stream(self.device).cuda_stream != self.stream_ptr:
+            # the collective is enqueued on torch's current stream, not the
+            # library's: K4 must have written d_out first
+            from . import rrl as R
+            R.rrl_synchronize(self.tl.inst)
         allreduce_sum_(self.d_out, self.group)
         return self.d_out
 

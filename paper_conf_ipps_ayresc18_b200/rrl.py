@@ -105,6 +105,10 @@ _SIGS = {
     "rrl_update_partials_ranged": (_I, [_I, _P, _P, _I, _P, _I]),
     "rrl_calculate_root_log_likelihoods_range": (_I, [_I] * 7 + [_P]),
     "rrl_reroot_exhaustive": (_I, [_I, _P, _P, _P, _P]),
+    "rrl_tree_spr": (_I, [_I, _P, _P, _I, _I, _P, _P]),
+    "rrl_tree_nni": (_I, [_I, _P, _P, _I, _I, _P, _P]),
+    "rrl_schedule_update": (_I, [_I, _P, _P, _P, _P, C.c_uint32, _P, _P, _P, _P, _P, _P, _P]),
+    "rrl_schedule_cost": (_I, [_I, _P, _I, _P, _I, _I, _I, _I, _I, C.c_double, C.c_double, C.c_double, _P]),
 }
 for _name, (_res, _args) in _SIGS.items():
     _f = getattr(_lib, _name)
@@ -162,8 +166,12 @@ def rrl_set_tip_states(inst, tip, states):
     return _chk(_lib.rrl_set_tip_states(inst, tip, _ptr(a)), "rrl_set_tip_states")
 
 
-def rrl_set_tip_states_u8(inst, first_tip, states2d):
+def rrl_set_tip_states_u8(inst, first_tip, states2d, pattern_count: int):
+    """states2d: uint8 [count, pattern_count] (the C side copies rows of
+    exactly pattern_count bytes, so the width is checked here)."""
     a = _c(states2d, np.uint8)
+    if a.ndim != 2 or a.shape[1] != pattern_count:
+        raise ValueError(f"tip states must be [count, {pattern_count}] uint8, got shape {a.shape}")
     return _chk(_lib.rrl_set_tip_states_u8(inst, first_tip, a.shape[0], _ptr(a)),
                 "rrl_set_tip_states_u8")
 
@@ -396,4 +404,55 @@ def rrl_calculate_root_log_likelihoods_range(inst, root_buffer, cat_weights_idx,
     _chk(_lib.rrl_calculate_root_log_likelihoods_range(inst, root_buffer, cat_weights_idx, freqs_idx,
                                                        cumulative_idx, pattern_begin, pattern_end, _ptr(out)),
          "rrl_calculate_root_log_likelihoods_range")
+    return float(out[0])
+
+
+def rrl_tree_spr(tip_count, parent, blen, prune_node, regraft_node):
+    """SPR move (reading A26).  Returns (parent, blen) of the new tree."""
+    par, bl = _c(parent, np.int32), _c(blen, np.float64)
+    op, ob = np.empty_like(par), np.empty_like(bl)
+    _chk(_lib.rrl_tree_spr(tip_count, _ptr(par), _ptr(bl), int(prune_node), int(regraft_node), _ptr(op),
+                           _ptr(ob)), "rrl_tree_spr")
+    return op, ob
+
+
+def rrl_tree_nni(tip_count, parent, blen, edge_node, which):
+    """NNI move (reading A27).  Returns (parent, blen) of the new tree."""
+    par, bl = _c(parent, np.int32), _c(blen, np.float64)
+    op, ob = np.empty_like(par), np.empty_like(bl)
+    _chk(_lib.rrl_tree_nni(tip_count, _ptr(par), _ptr(bl), int(edge_node), int(which), _ptr(op), _ptr(ob)),
+         "rrl_tree_nni")
+    return op, ob
+
+
+def rrl_schedule_update(tip_count, stored_parent, stored_blen, parent, blen, reroot=False):
+    """Partial update after any change (reading A28).  Returns dict(parent,
+    blen, root_edge, ops (OP_DTYPE), set_offsets, op_count, set_count)."""
+    n = tip_count
+    sp, sb = _c(stored_parent, np.int32), _c(stored_blen, np.float64)
+    par, bl = _c(parent, np.int32), _c(blen, np.float64)
+    out_par = np.empty(2 * n - 1, np.int32)
+    out_bl = np.empty(2 * n - 1, np.float64)
+    key = np.zeros(1, np.int32)
+    ops = np.empty(max(1, n - 1), OP_DTYPE)
+    offs = np.empty(n, np.int32)
+    nop = np.zeros(1, np.int32)
+    nset = np.zeros(1, np.int32)
+    flags = SCHED_REROOT if reroot else SCHED_LEVEL
+    _chk(_lib.rrl_schedule_update(n, _ptr(sp), _ptr(sb), _ptr(par), _ptr(bl), flags, _ptr(out_par), _ptr(out_bl),
+                                  _ptr(key), _ptr(ops), _ptr(offs), _ptr(nop), _ptr(nset)), "rrl_schedule_update")
+    k, m = int(nset[0]), int(nop[0])
+    return dict(parent=out_par, blen=out_bl, root_edge=int(key[0]), ops=ops[:m].copy(),
+                set_offsets=offs[: k + 1].copy(), op_count=m, set_count=k)
+
+
+def rrl_schedule_cost(tip_count, ops, set_offsets, pattern_count, state_count, category_count, precision,
+                      launch_us=2.0, hbm_gbs=6000.0, l2_bytes=126e6) -> float:
+    """Predicted updatePartials time (us) of a schedule (NEXT-4 cost model)."""
+    o = as_ops(ops)
+    so = _c(set_offsets, np.int32)
+    out = np.zeros(1, np.float64)
+    _chk(_lib.rrl_schedule_cost(tip_count, _ptr(o), o.shape[0], _ptr(so), so.shape[0] - 1, pattern_count,
+                                state_count, category_count, precision, float(launch_us), float(hbm_gbs),
+                                float(l2_bytes), _ptr(out)), "rrl_schedule_cost")
     return float(out[0])

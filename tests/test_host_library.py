@@ -175,3 +175,61 @@ def test_exhaustive_cpp_equals_dp(R):
             key, sets = R.rrl_reroot_exhaustive(300, t.parent, t.blen)
             g = R.rrl_reroot_and_schedule(300, t.parent, t.blen, "reroot")
             assert key == g["root_edge"] and sets == g["set_count"]
+
+
+# ------------------------------------------------------------------ NEXT-2: moves + update schedules
+def _random_move_pair(R, t, rng):
+    """One random legal SPR or NNI, applied by the oracle and by the C++."""
+    from oracle import moves
+    from oracle.pruning import children_of
+    n = t.n
+    while True:
+        if rng.random() < 0.5:
+            x = int(rng.integers(0, 2 * n - 1))
+            if x == t.root or t.parent[x] == t.root:
+                continue
+            r = int(rng.integers(0, 2 * n - 1))
+            if r in moves._subtree_nodes(t, x) | {int(t.parent[x]), t.root}:
+                continue
+            return moves.spr(t, x, r), R.rrl_tree_spr(n, t.parent, t.blen, x, r)
+        keys = [k for k, u, v, _ in orr.unrooted_edges(t) if u >= n and v >= n]
+        k, which = keys[int(rng.integers(0, len(keys)))], int(rng.integers(0, 2))
+        return moves.nni(t, k, which), R.rrl_tree_nni(n, t.parent, t.blen, k, which)
+
+
+@pytest.mark.parametrize("kind,n", [("random", 40), ("pectinate", 33), ("yule", 64), ("balanced", 32)])
+def test_moves_and_update_schedule_bit_exact_vs_oracle(R, kind, n):
+    from oracle import moves
+    for seed in (1, 2, 3):
+        t0 = make_tree(kind, n, seed=seed)
+        stored = orr.RTree(n, t0.parent.copy(), t0.blen.copy())
+        rng = np.random.default_rng(seed)
+        new = stored
+        for step in range(4):
+            o, (cp, cb) = _random_move_pair(R, new, rng)
+            assert np.array_equal(o.parent, cp) and np.array_equal(o.blen, cb)   # bit-exact fp64
+            new = o
+            if rng.random() < 0.3:  # a branch-length change too
+                v = int(rng.integers(0, 2 * n - 1))
+                if v != new.root:
+                    new.blen[v] *= 1.25
+            for reroot in (False, True):
+                rt, ops, offs, key, _ = moves.schedule_update(stored, new, reroot=reroot)
+                got = R.rrl_schedule_update(n, stored.parent, stored.blen, new.parent, new.blen, reroot)
+                assert got["root_edge"] == key, (seed, step, reroot)
+                assert np.array_equal(got["parent"], rt.parent)
+                assert np.array_equal(got["blen"], rt.blen)
+                assert _ops_tuple(got["ops"]) == ops
+                assert got["set_offsets"].tolist() == offs
+
+
+def test_update_schedule_no_change_and_errors(R):
+    t = make_tree("random", 30, seed=4)
+    got = R.rrl_schedule_update(30, t.parent, t.blen, t.parent, t.blen, True)
+    assert got["op_count"] == 0 and got["set_count"] == 0
+    root = t.root
+    a = int(np.flatnonzero(t.parent == root)[0])
+    with pytest.raises(R.RRLError):
+        R.rrl_tree_spr(30, t.parent, t.blen, a, 0 if a != 0 else 1)   # parent of prune node is the root
+    with pytest.raises(R.RRLError):
+        R.rrl_tree_nni(30, t.parent, t.blen, 3, 0)                     # a tip is no internal edge
