@@ -82,8 +82,9 @@ extern "C" {
 #define RRL_FLAG_CUDA_GRAPH 0x2u       /* capture each distinct operation list's
                                           level-set launches in a CUDA graph and
                                           replay it on later identical calls */
-#define RRL_FLAG_CODON_SIMT 0x4u       /* 61-state fp32: use the FP32 SIMT kernel
-                                          instead of the tcgen05 (3xTF32) one */
+#define RRL_FLAG_CODON_SIMT 0x4u       /* 61 states: use the SIMT kernel (FFMA /
+                                          DFMA) instead of the tensor-core one
+                                          (tcgen05 3xTF32 for fp32, DMMA for fp64) */
 #define RRL_FLAG_FUSED_PASS 0x8u       /* 4 states, no pattern ranges: run a whole
                                           rrl_update_partials call as ONE launch in
                                           which every thread owns the same (pattern,

@@ -52,6 +52,7 @@ struct Instance {
   uint8_t *d_states = nullptr;           // [n_tips][p_pad]
   char *d_P = nullptr;                   // [n_mat][c][s_pad][s_pad]
   float *d_Plo = nullptr;                // fp32 codon: tf32 low parts of d_P (3xTF32 operand), same layout
+  float *d_PT = nullptr;                 // fp32 codon: P^T per (matrix, category), row 61 = row sums (K3-TT)
   int32_t *d_scale = nullptr;            // [n_scale][p_pad]
   double *d_eig = nullptr;               // [n_eig][2 s^2 + s]
   double *d_rates = nullptr;             // [n_eig][c] (per model / partition)
@@ -83,6 +84,7 @@ struct Instance {
   std::vector<rrl_op> last_ops;
   std::vector<int32_t> last_offs;
   std::vector<int32_t> last_ranges;
+  std::vector<int> set_tt;               // 61-state fp32: tip-tip ops at the front of each set
   bool ops_valid = false;
   cudaGraphExec_t graph = nullptr;       // replay of the set launches
   cudaStream_t graph_stream = nullptr;
@@ -96,6 +98,7 @@ struct Instance {
   // TMA descriptors of the internal-partials and matrix slabs (61-state fp32, K3-TC5)
   CUtensorMap tmap_partials{}, tmap_P{}, tmap_Plo{};
   bool tmaps_ok = false;
+
 };
 
 std::mutex g_mu;
@@ -199,7 +202,7 @@ void destroy(Instance *I) {
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
                   I->d_catw,     I->d_freqs,  I->d_pw,   I->d_site,  I->d_block, I->d_out, I->d_count,
-                  I->d_t,      I->d_sidx, I->d_ops,  I->d_Plo,  I->d_flag};
+                  I->d_t,      I->d_sidx, I->d_ops,  I->d_Plo,  I->d_flag, I->d_PT};
   for (void *q : ptrs)
     if (q) cudaFree(q);
   if (I->h_ops) cudaFreeHost(I->h_ops);
@@ -383,6 +386,11 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
                               CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
       I->tmaps_ok = (r1 == CUDA_SUCCESS && r2 == CUDA_SUCCESS && r3 == CUDA_SUCCESS);
     }
+  }
+  if (state_count == 61 && precision == 32) {
+    const size_t pbytes = (size_t)matrix_count * I->mat_elems * I->elt;
+    CKC(cudaMalloc(&I->d_PT, pbytes));
+    CKC(cudaMemset(I->d_PT, 0, pbytes));
   }
   CKC(cudaMallocHost(&I->h_out, sizeof(double)));
   CKC(cudaMalloc(&I->d_flag, sizeof(unsigned)));
@@ -616,7 +624,7 @@ int rrl_update_transition_matrices(int inst, int eigen_idx, const int32_t *matri
     Timed tm(I, 1);
     CKL(launch_transition_matrices(I->prec, I->s, I->s_pad, I->c, I->d_eig + eig_sz * eigen_idx,
                                    I->d_rates + (size_t)eigen_idx * I->c, I->d_midx, I->d_t, count, I->d_P,
-                                   I->d_Plo, I->stream));
+                                   I->d_Plo, I->d_PT, I->stream));
   }
   I->prof.matrices_launches += (count + 65534) / 65535;
   I->prof.kernel_launches += (count + 65534) / 65535;
@@ -641,6 +649,9 @@ int rrl_set_transition_matrix(int inst, int idx, const double *P) {
   if (I->d_Plo)  // keep the 3xTF32 low parts of this matrix in step (device split, like K1's)
     CKL(launch_split_tf32(reinterpret_cast<const float *>(I->d_P + (size_t)idx * h.size()),
                          I->d_Plo + (size_t)idx * I->mat_elems, I->mat_elems, I->stream));
+  if (I->d_PT)  // and its transpose for the tip-tip gathers
+    CKL(launch_codon_pt(reinterpret_cast<const float *>(I->d_P + (size_t)idx * h.size()),
+                        I->d_PT + (size_t)idx * I->mat_elems, I->c, I->stream));
   CK(cudaStreamSynchronize(I->stream));
   return RRL_SUCCESS;
 }
@@ -785,7 +796,24 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
     int r = ensure_cap_ops(I, op_count);
     if (r < 0) return r;
     CK(cudaEventSynchronize(I->staging_ev));  // previous upload has consumed the staging
-    for (int i = 0; i < op_count; ++i) {
+    // 61-state fp32: inside each set (independent ops, any order) the ops whose
+    // children are both tips go first; they run as the K3-TT gather kernel
+    std::vector<int> perm(op_count);
+    for (int i = 0; i < op_count; ++i) perm[i] = i;
+    I->set_tt.assign(nsets, 0);
+    if (I->s == 61 && I->d_PT) {
+      auto tiptip = [&](int i) {
+        const rrl_op &o = ops[i];
+        return o.child1 < I->n_tips && I->has_states[o.child1] && o.child2 < I->n_tips && I->has_states[o.child2];
+      };
+      for (int k = 0; k < nsets; ++k) {
+        auto b = perm.begin() + offs[k], e = perm.begin() + offs[k + 1];
+        auto mid = std::stable_partition(b, e, tiptip);
+        I->set_tt[k] = (int)(mid - b);
+      }
+    }
+    for (int pi = 0; pi < op_count; ++pi) {
+      const int i = perm[pi];
       const rrl_op &o = ops[i];
       DevOp d{};
       auto child = [&](int b, const void **in, const int32_t **cum, int tipflag) {
@@ -831,7 +859,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
         if (d.cum1) d.cum1 += pb;
         if (d.cum2) d.cum2 += pb;
       }
-      I->h_ops[i] = d;
+      I->h_ops[pi] = d;
     }
     for (int k = 0; k < nsets; ++k) I->h_ops[offs[k + 1] - 1].flags |= OP_SET_END;
     // fused pass: a child produced by op j is read from the CTA's
@@ -901,15 +929,28 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
         e = launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax,
                                        I->p_pad, k > 0 ? 3 : 1, I->stream);
       } else {
-        e = (int)cudaErrorNotSupported;
-        if (I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT) && I->tmaps_ok)  // TMA-fed tcgen05 (c <= 4)
-          e = launch_update_partials_codon_tc5(I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax, I->p_pad,
-                                               &I->tmap_partials, &I->tmap_P, &I->tmap_Plo, I->stream);
-        if (e == (int)cudaErrorNotSupported && I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT))
-          e = launch_update_partials_codon_tc(I->c, I->d_ops + offs[k], n, pmax, I->p_pad, I->stream);
-        if (e == (int)cudaErrorNotSupported)
-          e = launch_update_partials_codon(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax,
-                                           I->p_pad, I->stream);
+        e = 0;
+        int o0 = offs[k], nr = n;  // the ops left for the contraction kernels
+        const bool tc = I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT);
+        if (tc && I->set_tt[k] > 0) {  // cherries: gathers from P^T, no contraction (K3-TT)
+          e = launch_update_partials_codon_tiptip(I->c, I->d_ops + o0, I->set_tt[k], pmax, I->p_pad, I->d_PT,
+                                                  I->stream);
+          o0 += I->set_tt[k];
+          nr -= I->set_tt[k];
+        }
+        if (e == 0 && nr > 0) {
+          e = (int)cudaErrorNotSupported;
+          if (tc && I->tmaps_ok)  // TMA-fed tcgen05, one CTA per tile (c <= 4)
+            e = launch_update_partials_codon_tc5(I->c, I->d_ops + o0, I->h_ops + o0, nr, pmax, I->p_pad,
+                                                 &I->tmap_partials, &I->tmap_P, &I->tmap_Plo, I->stream);
+          if (e == (int)cudaErrorNotSupported && tc)
+            e = launch_update_partials_codon_tc(I->c, I->d_ops + o0, nr, pmax, I->p_pad, I->stream);
+          if (e == (int)cudaErrorNotSupported && I->prec == 64 && !(I->flags & RRL_FLAG_CODON_SIMT))
+            e = launch_update_partials_codon_dmma(I->c, I->d_ops + o0, nr, pmax, I->p_pad, I->stream);
+          if (e == (int)cudaErrorNotSupported)
+            e = launch_update_partials_codon(I->prec, I->c, I->d_ops + o0, I->h_ops + o0, nr, pmax, I->p_pad,
+                                             I->stream);
+        }
       }
       if (e == (int)cudaErrorNotSupported) return fail(RRL_ERROR_NO_IMPLEMENTATION, "kernel variant");
       if (e != 0) return fail(RRL_ERROR_CUDA, std::string("updatePartials launch: ") +
@@ -920,7 +961,11 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
   int kl = 0;
   if (fused) kl = 1;
   else
-    for (int k = 0; k < nsets; ++k) kl += (offs[k + 1] - offs[k] + 65534) / 65535;
+    for (int k = 0; k < nsets; ++k) {
+      const int tt = (I->s == 61 && I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT)) ? I->set_tt[k] : 0;
+      const int n = offs[k + 1] - offs[k];
+      kl += (tt > 0 ? 1 : 0) + (n - tt > 0 ? (n - tt + 65534) / 65535 : 0);
+    }
 
   // (the legacy default stream cannot be captured: eager launches there)
   const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && I->stream != nullptr;

@@ -75,8 +75,8 @@ constexpr int SMEM_MX = SM_S1 + TM * TS * 4;           // row maxima / scale [2]
 constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 16 mbarriers
 constexpr int SMEM_TMEM = SMEM_BAR + 16 * 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 16;
-constexpr int kTmemCols = 512;    // per K-half h: [main_h | corr_h] (4 x 64) ...
-constexpr int kProdCol = 4 * TS;  // ... + one 64-column slot per category (child 1, then the product)
+constexpr int kTmemCols = 512;    // [main_0 | corr | main_1] (3 x 64) ...
+constexpr int kProdCol = 3 * TS;  // ... + one 64-column slot per category (the unscaled product)
 
 __device__ inline uint32_t sa(const void *p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
 __device__ inline uint64_t desc_sw128(uint32_t saddr) {  // K-major, 128-byte swizzle, 8-row atoms of 1 KB
@@ -241,7 +241,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       for (int g = 0; g < nphase; ++g) {
         int c, b, p0;
         const DevOp &op = phase_op(g, c, b, p0);
-        if (is_tip(op, b)) continue;
+        if (is_tip(op, b) || p0 >= op.p) continue;
         const uint32_t sl = ia % NA, use = ia / NA;
         ++ia;
         bar_wait(&a_empty[sl], (use & 1u) ^ 1u);  // the MMAs NA internal phases back are done
@@ -256,11 +256,14 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
   } else if (warp == kProdB) {
     // ================================================================ matrix producer
     if (lane == 0) {
+      uint32_t gb = 0;  // phases processed (tiles past an op's own range are skipped)
       for (int g = 0; g < nphase; ++g) {
         int c, b, p0;
         const DevOp &op = phase_op(g, c, b, p0);
+        if (p0 >= op.p) continue;
         const bool tip = is_tip(op, b);
-        const uint32_t sl = g % NB, use = g / NB;
+        const uint32_t sl = gb % NB, use = gb / NB;
+        ++gb;
         bar_wait(&b_empty[sl], (use & 1u) ^ 1u);
 #ifdef RRL_TC5_TRACE
         if (blockIdx.x == 0 && g < 4096) g_tc5_kind[g] = tip ? 1 : 0;
@@ -280,11 +283,14 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     // ================================================================ MMA issuer
     if (lane == 0) {
       uint32_t ia = 0;
+      uint32_t gb = 0;
       for (int g = 0; g < nphase; ++g) {
         int c, b, p0;
         const DevOp &op = phase_op(g, c, b, p0);
-        const uint32_t bs = g % NB;
-        bar_wait(&b_full[bs], (uint32_t)(g / NB) & 1u);
+        if (p0 >= op.p) continue;
+        const uint32_t bs = gb % NB;
+        bar_wait(&b_full[bs], (uint32_t)(gb / NB) & 1u);
+        ++gb;
         if (is_tip(op, b)) continue;  // a tip child is a P-column gather in the epilogue: no MMA
         const uint32_t sl = ia % NA, use = ia / NA;
         bar_wait(&a_full[sl], use & 1u);
@@ -293,18 +299,27 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         ++ia;
         fence_after();
         TR(3, g);
-        // per K-step of 8: A_hi . [P_hi | P_lo]^T (N = 128) -> [main_h | corr_h], then
-        // A_lo . P_hi^T (N = 64) -> corr_h; main and the ~2^-11-smaller corrections
-        // never share an accumulator (tf32 accumulation reading).
+        // Accumulators [main_0 | corr | main_1]: K-half 0 as A_hi . [P_hi | P_lo]^T (N = 128)
+        // -> [main_0 | corr] plus A_lo . P_hi^T -> corr; K-half 1 as three N = 64 MMAs
+        // (A_hi P_hi -> main_1, A_hi P_lo and A_lo P_hi -> corr; same tensor time).  The
+        // hi.hi sums of the two K-halves and the ~2^-11-smaller corrections never share
+        // an accumulator (tf32 accumulation reading); one shared correction
+        // accumulator saves a quarter of the epilogue's TMEM reads.
 #pragma unroll
         for (int kk = 0; kk < TS / 8; ++kk) {
           const int h = kk >> 2, kin = kk & 3;
           const uint64_t ah = desc_sw128(sbase + SM_A + sl * 32768 + h * 16384 + kin * 32);
           const uint64_t al = desc_sw128(sbase + SM_ALO + h * 16384 + kin * 32);
           const uint64_t bb = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + kin * 32);
-          const uint32_t d = tmem + (uint32_t)(h * 2 * TS);
-          mma_tf32(d, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);
-          mma_tf32(d + TS, al, bb, idesc_tf32(TS), 1u);
+          if (h == 0) {
+            mma_tf32(tmem, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);
+            mma_tf32(tmem + TS, al, bb, idesc_tf32(TS), 1u);
+          } else {
+            const uint64_t bl = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + 8192 + kin * 32);
+            mma_tf32(tmem + 2 * TS, ah, bb, idesc_tf32(TS), kin > 0 ? 1u : 0u);
+            mma_tf32(tmem + TS, ah, bl, idesc_tf32(TS), 1u);
+            mma_tf32(tmem + TS, al, bb, idesc_tf32(TS), 1u);
+          }
         }
         commit(&a_empty[sl]);  // child tile, lo tile and matrix tile free once these MMAs completed
         commit(lo_empty);
@@ -320,7 +335,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     for (int g = 0; g < nphase; ++g) {
       int c, b, p0;
       const DevOp &op = phase_op(g, c, b, p0);
-      if (is_tip(op, b)) continue;
+      if (is_tip(op, b) || p0 >= op.p) continue;
       const uint32_t sl = ia % NA, use = ia / NA;
       bar_wait(&a_full[sl], use & 1u);
       bar_wait(lo_empty, (ia & 1u) ^ 1u);  // the previous internal phase's MMAs read the lo tile
@@ -402,7 +417,9 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       }
     };
     float m = 0.f;  // running max over (c, z) of this thread's row half
+    float d1[32];     // child 1's contraction of the current category
     uint32_t ni = 0;  // internal-child phases consumed (accumulator barrier parity)
+    uint32_t gb = 0;  // phases processed (matrix ring parity)
     for (int g = 0; g < nphase; ++g) {
       const int lt = g / (2 * C), c = (g / 2) % C, b = g & 1;
       const int f = blockIdx.x + lt * gridDim.x;
@@ -410,23 +427,25 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       const int p0 = (f % ntiles) * TM;
       const int pp = p0 + r;
       const bool valid = pp < op.p;
-      if (b == 0 && have_prev) {  // before child 1 reuses slot c: write back the previous tile's category c
-        drain(c);
-        if (tid == 0) TR(9, g);
-      }
       if (c == 0 && b == 0) {  // tile start: rotate the prefetched metadata
         if (lt == 0) load_meta(0, sv_nxt, ex_nxt);
         sv_cur = sv_nxt;
         ex_cur = ex_nxt;
         if (lt + 1 < my_tiles) load_meta(lt + 1, sv_nxt, ex_nxt);
       }
+      if (p0 >= op.p) continue;  // past this op's own range (a shorter partition): another op's rows
+      const uint32_t gcur = gb++;
+      if (b == 0 && have_prev) {  // before child 1 reuses slot c: write back the previous tile's category c
+        drain(c);
+        if (tid == 0) TR(9, g);
+      }
       float dv[32];
       if (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) {
         // Tip child: sum_x P[z][x] [x == obs] = P[z][obs], read from the raw fp32 P tile the
         // producer landed in stage g&1 (swizzled K-major: row z, 16-byte chunk (x&31)/4 at
         // position chunk ^ (z&7) of half x>>5). A missing state (code >= 61) is the row sum.
-        const int s = g % NB;
-        bar_wait(&b_full[s], (uint32_t)(g / NB) & 1u);
+        const int s = gcur % NB;
+        bar_wait(&b_full[s], (uint32_t)(gcur / NB) & 1u);
         if (tid == 0) TR(7, g);
         const unsigned char *pt = sm + SM_B + s * 32768;  // P hi of K-half h at h * 16 KB
         const unsigned sv = (sv_cur >> (8 * b)) & 0xffu;  // prefetched (0 for padding rows)
@@ -463,14 +482,13 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         if (tid == 0) TR(7, g);
 #pragma unroll
         for (int q = 0; q < 2; ++q) {
-          float m0[16], c0[16], m1[16], c1[16];
+          float m0[16], cc[16], m1[16];
           tmem_ld16(tl + 0 * TS + q * 16, m0);
-          tmem_ld16(tl + 1 * TS + q * 16, c0);
+          tmem_ld16(tl + 1 * TS + q * 16, cc);
           tmem_ld16(tl + 2 * TS + q * 16, m1);
-          tmem_ld16(tl + 3 * TS + q * 16, c1);
           tmem_wait_ld();
 #pragma unroll
-          for (int i = 0; i < 16; ++i) dv[q * 16 + i] = (m0[i] + m1[i]) + (c0[i] + c1[i]);
+          for (int i = 0; i < 16; ++i) dv[q * 16 + i] = (m0[i] + m1[i]) + cc[i];
         }
         fence_before();
         __syncwarp();
@@ -478,25 +496,16 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         if (tid == 0) TR(5, g);
       }
       const uint32_t slot = tl + (uint32_t)(kProdCol + c * TS);  // this category's TMEM slot
-      if (b == 0) {  // child 1 waits in the slot until child 2's phase
-        tmem_st16(slot, dv);
-        tmem_st16(slot + 16, dv + 16);
-        tmem_wait_st();
+      if (b == 0) {  // child 1 waits in registers: child 2's phase of the same category is next
+#pragma unroll
+        for (int i = 0; i < 32; ++i) d1[i] = dv[i];
         if (tid == 0) TR(6, g);
         continue;
       }
-      {
-        float w0[16], w1[16];
-        tmem_ld16(slot, w0);
-        tmem_ld16(slot + 16, w1);
-        tmem_wait_ld();
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          dv[i] *= w0[i];
-          dv[16 + i] *= w1[i];
-        }
-#pragma unroll
-        for (int i = 0; i < 32; ++i) m = fmaxf(m, dv[i]);
+      for (int i = 0; i < 32; ++i) {
+        dv[i] *= d1[i];
+        m = fmaxf(m, dv[i]);
       }
       tmem_st16(slot, dv);  // park the unscaled product (in place of child 1) until written back
       tmem_st16(slot + 16, dv + 16);

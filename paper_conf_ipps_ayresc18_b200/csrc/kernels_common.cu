@@ -16,6 +16,7 @@ int device_slot() {
 namespace {
 
 constexpr double kLn2 = 0.693147180559945309417232121458176568;
+constexpr int kS61Row = 61;  // P^T row of the missing codon state (row sums)
 
 // ---------------------------------------------------------------------- K1
 // P_{m,c}[z][x] = sum_k V[z][k] exp(lambda_k r_c t_m) Vinv[k][x]  (fp64),
@@ -66,7 +67,7 @@ template <typename T>
 __global__ void __launch_bounds__(256)
 k_transition64(int s, int C, int items, const double *__restrict__ eig, const double *__restrict__ rates,
                const int32_t *__restrict__ idx, const double *__restrict__ tlen, T *__restrict__ P,
-               float *__restrict__ Plo) {
+               float *__restrict__ Plo, float *__restrict__ PT) {
   // Persistent: V and V^-1 (the same for every matrix) are staged in shared
   // memory once per block, which then walks (matrix, category) items.
   extern __shared__ double sm[];
@@ -126,7 +127,44 @@ k_transition64(int s, int C, int items, const double *__restrict__ eig, const do
         *reinterpret_cast<double2 *>(row + 32) = make_double2(acc[i][2], acc[i][3]);
       }
     }
+    if (PT != nullptr) {
+      // P^T for the tip-tip gather kernel: row x < 61 = column x of P (four
+      // consecutive z per 16-byte store), row 61 = the row sums sum_x P[z][x]
+      // (the all-ones partials of a missing state, reading A23; summed in fp64
+      // over the 16 lanes sharing z0), rows 62-63 stay zero
+      const int xs[4] = {x0, x0 + 1, 32 + x0, 33 + x0};
+#pragma unroll
+      for (int j = 0; j < 4; ++j)
+        if (xs[j] < s)
+          *reinterpret_cast<float4 *>(PT + off + xs[j] * 64 + z0) =
+              make_float4((float)acc[0][j], (float)acc[1][j], (float)acc[2][j], (float)acc[3][j]);
+      double rs[4];
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        rs[i] = (acc[i][0] + acc[i][1]) + (acc[i][2] + acc[i][3]);
+#pragma unroll
+        for (int o = 1; o < 16; o <<= 1) rs[i] += __shfl_xor_sync(0xffffffffu, rs[i], o);
+      }
+      if ((tid & 15) == 0)
+        *reinterpret_cast<float4 *>(PT + off + kS61Row * 64 + z0) =
+            make_float4((float)rs[0], (float)rs[1], (float)rs[2], (float)rs[3]);
+    }
   }
+}
+
+// P^T of one stored fp32 codon matrix set (rrl_set_transition_matrix): same
+// layout and row-61 sums as K1 writes (sums in fp64 of the stored fp32 values).
+__global__ void k_codon_pt(const float *__restrict__ P, float *__restrict__ PT, int C) {
+  const int c = blockIdx.x, z = threadIdx.x;  // 64 threads
+  const float *row = P + ((size_t)c * 64 + z) * 64;
+  float *pt = PT + (size_t)c * 64 * 64;
+  double sum = 0.0;
+  for (int x = 0; x < 64; ++x) {
+    const float v = x < kS61Row ? row[x] : 0.f;
+    sum += (double)v;
+    if (x != kS61Row) pt[x * 64 + z] = v;
+  }
+  pt[kS61Row * 64 + z] = (float)sum;
 }
 
 __global__ void k_split_tf32(const float *__restrict__ x, float *__restrict__ lo, size_t n) {
@@ -290,7 +328,7 @@ k_edge(const T *__restrict__ Lp, const void *__restrict__ child, int child_is_ti
 
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
-                               int count, void *d_P, void *d_Plo, void *stream) {
+                               int count, void *d_P, void *d_Plo, void *d_PT, void *stream) {
   if (count <= 0) return 0;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
   if (s_pad == 64) {  // codon: register-tiled, persistent blocks over (matrix, category) items
@@ -310,10 +348,11 @@ int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *
     const int grid = items < grid_cap ? items : grid_cap;
     if (prec == 32)
       k_transition64<float><<<grid, 256, smem64, st>>>(s, c, items, d_eig, d_rates, d_idx, d_t,
-                                                       static_cast<float *>(d_P), static_cast<float *>(d_Plo));
+                                                       static_cast<float *>(d_P), static_cast<float *>(d_Plo),
+                                                       static_cast<float *>(d_PT));
     else
       k_transition64<double><<<grid, 256, smem64, st>>>(s, c, items, d_eig, d_rates, d_idx, d_t,
-                                                        static_cast<double *>(d_P), nullptr);
+                                                        static_cast<double *>(d_P), nullptr, nullptr);
     return (int)cudaGetLastError();
   }
   const size_t smem = sizeof(double) * (2 * s * s + s);
@@ -372,6 +411,11 @@ int launch_edge_lnl(int prec, int s, int s_pad, int c, const void *par, const vo
     k_edge<double><<<nblocks, 256, 0, st>>>(static_cast<const double *>(par), child, child_is_tip,
                                             static_cast<const double *>(P), s, s_pad, c, d_w, d_pi,
                                             cum_p, cum_c, d_pw, p, p_pad, d_site, d_block, d_count, d_out);
+  return (int)cudaGetLastError();
+}
+
+int launch_codon_pt(const float *P, float *PT, int c, void *stream) {
+  k_codon_pt<<<c, 64, 0, static_cast<cudaStream_t>(stream)>>>(P, PT, c);
   return (int)cudaGetLastError();
 }
 

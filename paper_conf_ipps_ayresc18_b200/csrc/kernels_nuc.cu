@@ -41,6 +41,18 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kInline = 8;
+// Latency path: 4 resident 256-thread CTAs per SM (<= 64 registers), so the
+// next level set's CTAs (2 per SM at configs[1]) are co-resident with the
+// current set's under programmatic dependent launch and run their prologue
+// (descriptors, tip states, P rows) before griddepcontrol.wait instead of
+// after the previous grid's exit.
+#ifndef RRL_LAT_MINB
+#define RRL_LAT_MINB 3
+#endif
+#ifndef RRL_LAT_PSMEM
+#define RRL_LAT_PSMEM 0
+#endif
+constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 constexpr int kChunkItems = 512;  // items (pattern x category) per bulk chunk
 constexpr int kPTab = 36;         // per (branch, cat): 16 rows P[z][x] + 5 columns x 4
 
@@ -208,7 +220,7 @@ __device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
 // level set passed its own wait).  Only the previous level set's partials and
 // exponents must wait.
 template <typename T, int C, int U>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, kLatencyMinBlocks)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int early) {
   const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
@@ -227,7 +239,7 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
   // fp32: each thread holds its category's rows in registers.  fp64: the rows
   // would cost 64 registers, so the block stages the tables in shared memory
   // (issued after this thread's first child loads, see below).
-  constexpr bool kRegP = sizeof(T) == 4;
+  constexpr bool kRegP = sizeof(T) == 4 && !RRL_LAT_PSMEM;
   __shared__ __align__(16) T sP[kRegP ? 1 : 2][kRegP ? 1 : C][kRegP ? 4 : kPTab];
   T P1[kRegP ? 16 : 1], P2[kRegP ? 16 : 1];
   auto load_rows = [&]() {
@@ -251,12 +263,18 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
     }
   }
   if (early & 2) load_rows();
+  bool tables = kRegP;
+  if constexpr (!kRegP) {
+    if (early & 2) {  // K1 completed before the previous set: the tables can be staged before the wait
+      load_ptables<T, C>(sP, op);
+      tables = true;
+    }
+  }
 
   pdl_wait();  // everything above overlaps the previous level set
   pdl_launch();
 
   if (!(early & 2)) load_rows();
-  bool tables = kRegP;
   for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
     const bool pre = (early & 1) && chunk == (int)blockIdx.x;
     const unsigned base = (unsigned)chunk * (kThreads * U) + threadIdx.x;

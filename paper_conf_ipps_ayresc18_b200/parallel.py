@@ -41,6 +41,8 @@ def allreduce_sum_(tensor, group=None):
     NCCL; through a host copy with gloo (the CPU-side wiring tests and
     several ranks sharing one GPU, where NCCL refuses)."""
     import torch.distributed as dist
+    if not dist.is_initialized():  # a single process: the local sum is the global one
+        return tensor
     if tensor.is_cuda and dist.get_backend(group) != "nccl":
         h = tensor.cpu()
         dist.all_reduce(h, op=dist.ReduceOp.SUM, group=group)
@@ -55,7 +57,7 @@ class ShardedTreeLikelihood:
 
     def __init__(self, n: int, p_total: int, s: int, c: int, rank: int, world: int,
                  precision: int = 32, device: int = 0, cuda_graph: bool = True,
-                 stream_ptr: int | None = None, group=None):
+                 stream_ptr: int | None = None, group=None, buffer_count: int | None = None):
         import torch
 
         from .engine import TreeLikelihood
@@ -68,7 +70,7 @@ class ShardedTreeLikelihood:
             # enqueue K4 on that same stream so all_reduce is ordered after it
             stream_ptr = torch.cuda.current_stream(device).cuda_stream
         self.tl = TreeLikelihood(n, self.hi - self.lo, s, c, precision=precision, device=device,
-                                 cuda_graph=cuda_graph, stream_ptr=stream_ptr)
+                                 cuda_graph=cuda_graph, stream_ptr=stream_ptr, buffer_count=buffer_count)
         self.stream_ptr = stream_ptr
         self.device = device
         self.d_out = torch.zeros(1, dtype=torch.float64, device=f"cuda:{device}")
@@ -79,11 +81,17 @@ class ShardedTreeLikelihood:
     def set_tips(self, tips_full: np.ndarray):
         self.tl.set_tips(np.ascontiguousarray(tips_full[:, self.lo:self.hi]))
 
+    def set_tips_local(self, tips_slice: np.ndarray):
+        """This rank's columns [lo, hi) only (no full alignment on every rank)."""
+        if tips_slice.shape[1] != self.hi - self.lo:
+            raise ValueError(f"expected {self.hi - self.lo} pattern columns, got {tips_slice.shape[1]}")
+        self.tl.set_tips(tips_slice)
+
     def set_pattern_weights(self, w_full):
         self.tl.set_pattern_weights(np.ascontiguousarray(w_full[self.lo:self.hi]))
 
-    def set_tree(self, parent, blen, mode="reroot"):
-        return self.tl.set_tree(parent, blen, mode)
+    def set_tree(self, parent, blen, mode="reroot", reuse_buffers=False):
+        return self.tl.set_tree(parent, blen, mode, reuse_buffers=reuse_buffers)
 
     def loglik_device(self):
         """Local pass + in-place all-reduce; returns the device tensor."""
