@@ -52,7 +52,7 @@ struct Instance {
   uint8_t *d_states = nullptr;           // [n_tips][p_pad]
   char *d_P = nullptr;                   // [n_mat][c][s_pad][s_pad]
   float *d_Plo = nullptr;                // fp32 codon: tf32 low parts of d_P (3xTF32 operand), same layout
-  float *d_PT = nullptr;                 // fp32 codon: P^T per (matrix, category), row 61 = row sums (K3-TT)
+  char *d_PT = nullptr;                  // codon: P^T per (matrix, category), row 61 = row sums (K3-TT)
   int32_t *d_scale = nullptr;            // [n_scale][p_pad]
   double *d_eig = nullptr;               // [n_eig][2 s^2 + s]
   double *d_rates = nullptr;             // [n_eig][c] (per model / partition)
@@ -72,6 +72,7 @@ struct Instance {
   int32_t *d_midx = nullptr;
   std::vector<char> h_tstage;  // host staging of the same layout: one H2D copy per call
   int t_cap = 0;
+  int t_count = -1;            // entries of h_tstage that mirror d_t (-1: none)
   // accumulate-scale index list
   int32_t *d_sidx = nullptr;
   int sidx_cap = 0;
@@ -387,7 +388,7 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
       I->tmaps_ok = (r1 == CUDA_SUCCESS && r2 == CUDA_SUCCESS && r3 == CUDA_SUCCESS);
     }
   }
-  if (state_count == 61 && precision == 32) {
+  if (state_count == 61) {
     const size_t pbytes = (size_t)matrix_count * I->mat_elems * I->elt;
     CKC(cudaMalloc(&I->d_PT, pbytes));
     CKC(cudaMemset(I->d_PT, 0, pbytes));
@@ -608,17 +609,26 @@ int rrl_update_transition_matrices(int inst, int eigen_idx, const int32_t *matri
     const size_t bytes = (sizeof(double) + sizeof(int32_t)) * (size_t)count;
     CK(cudaMalloc(&I->d_t, bytes));
     I->h_tstage.resize(bytes);
+    I->t_count = -1;
     I->d_midx = reinterpret_cast<int32_t *>(I->d_t + count);
     I->t_cap = count;
   }
   // [t | matrix_idx] packed, one H2D copy.  A copy from pageable memory is
   // staged by the driver before cudaMemcpyAsync returns, so neither the
-  // caller's arrays nor h_tstage are referenced after return.
+  // caller's arrays nor h_tstage are referenced after return.  The same
+  // branch lengths and indices as the previous call are already resident on
+  // the device (d_t is written only here): no copy.
   double *ht = reinterpret_cast<double *>(I->h_tstage.data());
-  std::memcpy(ht, t, sizeof(double) * count);
-  std::memcpy(ht + I->t_cap, matrix_idx, sizeof(int32_t) * count);
-  CK(cudaMemcpyAsync(I->d_t, ht, (sizeof(double) + sizeof(int32_t)) * (size_t)I->t_cap, cudaMemcpyHostToDevice,
-                     I->stream));
+  int32_t *hi = reinterpret_cast<int32_t *>(ht + I->t_cap);
+  const bool resident = count == I->t_count && std::memcmp(ht, t, sizeof(double) * count) == 0 &&
+                        std::memcmp(hi, matrix_idx, sizeof(int32_t) * count) == 0;
+  if (!resident) {
+    std::memcpy(ht, t, sizeof(double) * count);
+    std::memcpy(hi, matrix_idx, sizeof(int32_t) * count);
+    CK(cudaMemcpyAsync(I->d_t, ht, (sizeof(double) + sizeof(int32_t)) * (size_t)I->t_cap, cudaMemcpyHostToDevice,
+                       I->stream));
+    I->t_count = count;
+  }
   const size_t eig_sz = 2 * (size_t)I->s * I->s + I->s;
   {
     Timed tm(I, 1);
@@ -650,8 +660,8 @@ int rrl_set_transition_matrix(int inst, int idx, const double *P) {
     CKL(launch_split_tf32(reinterpret_cast<const float *>(I->d_P + (size_t)idx * h.size()),
                          I->d_Plo + (size_t)idx * I->mat_elems, I->mat_elems, I->stream));
   if (I->d_PT)  // and its transpose for the tip-tip gathers
-    CKL(launch_codon_pt(reinterpret_cast<const float *>(I->d_P + (size_t)idx * h.size()),
-                        I->d_PT + (size_t)idx * I->mat_elems, I->c, I->stream));
+    CKL(launch_codon_pt(I->prec, I->d_P + (size_t)idx * h.size(), I->d_PT + (size_t)idx * h.size(), I->c,
+                        I->stream));
   CK(cudaStreamSynchronize(I->stream));
   return RRL_SUCCESS;
 }
@@ -932,9 +942,10 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
         e = 0;
         int o0 = offs[k], nr = n;  // the ops left for the contraction kernels
         const bool tc = I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT);
-        if (tc && I->set_tt[k] > 0) {  // cherries: gathers from P^T, no contraction (K3-TT)
-          e = launch_update_partials_codon_tiptip(I->c, I->d_ops + o0, I->set_tt[k], pmax, I->p_pad, I->d_PT,
-                                                  I->stream);
+        const bool simt = (I->flags & RRL_FLAG_CODON_SIMT) != 0;
+        if (!simt && I->set_tt[k] > 0) {  // cherries: gathers from P^T, no contraction (K3-TT)
+          e = launch_update_partials_codon_tiptip(I->prec, I->c, I->d_ops + o0, I->set_tt[k], pmax, I->p_pad,
+                                                  I->d_PT, I->stream);
           o0 += I->set_tt[k];
           nr -= I->set_tt[k];
         }
@@ -946,7 +957,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
           if (e == (int)cudaErrorNotSupported && tc)
             e = launch_update_partials_codon_tc(I->c, I->d_ops + o0, nr, pmax, I->p_pad, I->stream);
           if (e == (int)cudaErrorNotSupported && I->prec == 64 && !(I->flags & RRL_FLAG_CODON_SIMT))
-            e = launch_update_partials_codon_dmma(I->c, I->d_ops + o0, nr, pmax, I->p_pad, I->stream);
+            e = launch_update_partials_codon_dmma(I->c, I->d_ops + o0, nr, pmax, I->p_pad, I->d_PT, I->stream);
           if (e == (int)cudaErrorNotSupported)
             e = launch_update_partials_codon(I->prec, I->c, I->d_ops + o0, I->h_ops + o0, nr, pmax, I->p_pad,
                                              I->stream);
@@ -962,7 +973,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
   if (fused) kl = 1;
   else
     for (int k = 0; k < nsets; ++k) {
-      const int tt = (I->s == 61 && I->prec == 32 && !(I->flags & RRL_FLAG_CODON_SIMT)) ? I->set_tt[k] : 0;
+      const int tt = (I->s == 61 && !(I->flags & RRL_FLAG_CODON_SIMT)) ? I->set_tt[k] : 0;
       const int n = offs[k + 1] - offs[k];
       kl += (tt > 0 ? 1 : 0) + (n - tt > 0 ? (n - tt + 65534) / 65535 : 0);
     }

@@ -19,10 +19,14 @@
 // B[t][g] (= P[8j + g][4k + t]), D[g][2t + i].  So a thread owns ONE pattern
 // (8w + g) and the 16 states 8j + 2t + i -- the tip gather and the per-pattern
 // max are per-thread work plus two xor-shuffles over the 4 lanes of a pattern.
-// Both operand tiles sit in shared memory with a 68-double row stride (a
-// warp's 32 LDS.64 of a fragment are two conflict-free wavefronts).  Each
-// category's unscaled product is stored at once with a running max kept; when
-// the max is known the thread rescales what it stored (L1/L2 hits).
+// The child tile of an internal child sits in shared memory (68-double rows:
+// a warp's 32 LDS.64 of a fragment are two conflict-free wavefronts),
+// double-buffered: the next internal stage is copied with cp.async while the
+// current stage's DMMAs run.  B fragments come straight from the 32 KB P tile
+// (L1-resident: every warp of the CTA reads it), and a tip child reads the
+// thread's 16 entries from row `state` of K1's P^T slab -- no staging, no
+// barrier.  Each category's unscaled product is stored at once with a running
+// max kept; when the max is known the thread rescales what it stored.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -33,12 +37,11 @@ namespace rrl {
 namespace {
 
 constexpr int kS = 61, kSP = 64, kTPD = 64, kThrD = 256;
-constexpr int kRow = 68;  // shared-memory row stride (doubles); column 64 of the P tile = row sums
+constexpr int kRow = 68;  // shared-memory row stride of the A tile (doubles)
 
 struct DmmaSmem {
-  double A[kTPD * kRow];  // child tile [pattern][x]
-  double P[kSP * kRow];   // the child's P [z][x], column 64 = sum_x P[z][x]
-  uint8_t st[2][kTPD];    // tip states of both children
+  double A[2][kTPD * kRow];  // double-buffered child tiles [pattern][x]
+  uint8_t st[2][kTPD];       // tip states of both children
 };
 
 __device__ inline void dmma(double (&d)[2], double a, double b) {
@@ -46,6 +49,13 @@ __device__ inline void dmma(double (&d)[2], double a, double b) {
                : "+d"(d[0]), "+d"(d[1])
                : "d"(a), "d"(b));
 }
+__device__ inline void cp_async16(void *smem, const void *gmem) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(static_cast<uint32_t>(__cvta_generic_to_shared(smem))),
+               "l"(gmem)
+               : "memory");
+}
+__device__ inline void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ inline void cp_async_wait_all() { asm volatile("cp.async.wait_group 0;" ::: "memory"); }
 __device__ inline int frexp_e64(double m) {
   const unsigned long long b = (unsigned long long)__double_as_longlong(m);
   const int eb = (int)((b >> 52) & 0x7ffull);
@@ -59,9 +69,12 @@ __device__ inline double pow2_neg64(int e) {
   return (e > -1022 && e < 1022) ? __longlong_as_double((long long)(1023 - e) << 52) : ldexp(1.0, -e);
 }
 
+// Stage (c, b) of a CTA = category c, child b; only internal children stage an
+// A tile.  The next internal stage's tile is copied (cp.async) into the other
+// buffer while the current stage's DMMAs run.
 template <int C>
 __global__ void __launch_bounds__(kThrD, 2)
-k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad) {
+k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__restrict__ PT) {
   extern __shared__ __align__(16) unsigned char smem_d[];
   DmmaSmem &sm = *reinterpret_cast<DmmaSmem *>(smem_d);
   const DevOp &op = ops[blockIdx.y];
@@ -71,6 +84,7 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad) {
   const bool tip[2] = {(op.flags & OP_TIP1) != 0, (op.flags & OP_TIP2) != 0};
   const void *in[2] = {op.in1, op.in2};
   const double *Pg[2] = {static_cast<const double *>(op.P1), static_cast<const double *>(op.P2)};
+  const int mat[2] = {op.mat1, op.mat2};
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, g = lane >> 2, t = lane & 3;
   const int prow = warp * 8 + g;  // this thread's pattern in the tile
   const int pp = p0 + prow;
@@ -78,6 +92,18 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad) {
 
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" :::);
+  auto stage_A = [&](int c, int b, int buf) {  // 64 rows x 512 B, 16-byte chunks; rows beyond p exist (p_pad)
+    const double *A = static_cast<const double *>(in[b]) + ((size_t)c * p_pad + p0) * kSP;
+    for (int i = tid; i < kTPD * kSP / 2; i += kThrD) {
+      const int r = i / 32, x2 = (i % 32) * 2;
+      cp_async16(&sm.A[buf][r * kRow + x2], A + 2 * i);
+    }
+    cp_async_commit();
+  };
+  // the internal stages in order: (c, b) for b with !tip[b]
+  const int nint = (tip[0] ? 0 : 1) + (tip[1] ? 0 : 1);
+  int si = 0;  // internal stages issued so far
+  if (nint > 0) stage_A(0, tip[0] ? 1 : 0, 0);
   for (int b = 0; b < 2; ++b)
     if (tip[b] && tid < kTPD) {
       const int q = p0 + tid;
@@ -87,49 +113,44 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad) {
   const double f_in = (!two_pass && op.scale_in != nullptr && valid) ? pow2_neg64(op.scale_in[pp]) : 1.0;
   double *out = static_cast<double *>(op.out);
   double m = 0.0;
+  __syncthreads();  // tip states
   for (int c = 0; c < C; ++c) {
     double d1[16];
+#pragma unroll
     for (int b = 0; b < 2; ++b) {
-      __syncthreads();  // the previous child's tiles are no longer read
-      const double *P = Pg[b] + (size_t)c * kSP * kSP;
-      for (int i = tid; i < kSP * kSP / 2; i += kThrD) {  // 16-byte chunks, coalesced
-        const int z = i / 32, x2 = (i % 32) * 2;
-        *reinterpret_cast<double2 *>(&sm.P[z * kRow + x2]) = __ldg(reinterpret_cast<const double2 *>(P) + i);
-      }
-      if (!tip[b]) {
-        const double *A = static_cast<const double *>(in[b]) + ((size_t)c * p_pad + p0) * kSP;
-        for (int i = tid; i < kTPD * kSP / 2; i += kThrD) {  // rows beyond p exist (p_pad)
-          const int r = i / 32, x2 = (i % 32) * 2;
-          *reinterpret_cast<double2 *>(&sm.A[r * kRow + x2]) = reinterpret_cast<const double2 *>(A)[i];
-        }
-      }
-      __syncthreads();
       double v[16];
       if (tip[b]) {
-        if (tid < kSP) {  // row sums: the all-ones partials of a missing state
-          double s = 0.0;
-          for (int x = 0; x < kS; ++x) s += sm.P[tid * kRow + x];
-          sm.P[tid * kRow + kSP] = s;
-        }
-        __syncthreads();
+        // P[z][s] for the thread's 16 states z = 8j + 2t + i: consecutive pairs of
+        // row s of P^T (K1; row 61 = row sums for a missing state), L1/L2-resident
         const unsigned s = sm.st[b][prow];
-        const int col = s < (unsigned)kS ? (int)s : kSP;
+        const double *row = PT + ((size_t)mat[b] * C + c) * kSP * kSP + (s < (unsigned)kS ? s : kS) * kSP + 2 * t;
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
-          v[2 * j] = sm.P[(8 * j + 2 * t) * kRow + col];
-          v[2 * j + 1] = sm.P[(8 * j + 2 * t + 1) * kRow + col];
+          const double2 x = __ldg(reinterpret_cast<const double2 *>(row + 8 * j));
+          v[2 * j] = x.x;
+          v[2 * j + 1] = x.y;
         }
       } else {
+        const int buf = si & 1;
+        cp_async_wait_all();
+        __syncthreads();  // this stage's tile landed for every thread; the other buffer is free
+        ++si;
+        if (si < nint * C) {  // prefetch the next internal stage
+          const int nb = (nint == 2) ? (b ^ 1) : b;
+          const int nc = (nint == 2) ? (b == 1 ? c + 1 : c) : c + 1;
+          stage_A(nc, nb, buf ^ 1);
+        }
         double acc[8][2];
 #pragma unroll
         for (int j = 0; j < 8; ++j) acc[j][0] = acc[j][1] = 0.0;
-        const double *Ar = &sm.A[prow * kRow + t];
-        const double *Pr = &sm.P[g * kRow + t];
+        const double *Ar = &sm.A[buf][prow * kRow + t];
+        // B fragment B[x][z] = P[z][x], z = 8j + g, x = 4k + t (L1-resident P tile)
+        const double *Pr = Pg[b] + (size_t)c * kSP * kSP + g * kSP + t;
 #pragma unroll 4
         for (int k = 0; k < kSP / 4; ++k) {
           const double a = Ar[4 * k];
 #pragma unroll
-          for (int j = 0; j < 8; ++j) dmma(acc[j], a, Pr[(8 * j) * kRow + 4 * k]);
+          for (int j = 0; j < 8; ++j) dmma(acc[j], a, __ldg(Pr + (8 * j) * kSP + 4 * k));
         }
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
@@ -181,7 +202,7 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad) {
 }
 
 template <int C>
-int launch_dmma(const DevOp *d_ops, int nops, int p, int p_pad, cudaStream_t st) {
+int launch_dmma(const DevOp *d_ops, int nops, int p, int p_pad, const double *PT, cudaStream_t st) {
   const size_t smem = sizeof(DmmaSmem);
   static bool configured_dev[kMaxDevices] = {};
   bool &configured = configured_dev[device_slot()];
@@ -204,7 +225,7 @@ int launch_dmma(const DevOp *d_ops, int nops, int p, int p_pad, cudaStream_t st)
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, k_partials_codon_dmma<C>, d_ops + o, p_pad);
+    cudaError_t e = cudaLaunchKernelEx(&cfg, k_partials_codon_dmma<C>, d_ops + o, p_pad, PT);
     if (e != cudaSuccess) return (int)e;
   }
   return 0;
@@ -212,13 +233,15 @@ int launch_dmma(const DevOp *d_ops, int nops, int p, int p_pad, cudaStream_t st)
 
 }  // namespace
 
-int launch_update_partials_codon_dmma(int c, const DevOp *d_ops, int nops, int p, int p_pad, void *stream) {
+int launch_update_partials_codon_dmma(int c, const DevOp *d_ops, int nops, int p, int p_pad, const void *d_PT,
+                                      void *stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  const double *PT = static_cast<const double *>(d_PT);
   switch (c) {
-    case 1: return launch_dmma<1>(d_ops, nops, p, p_pad, st);
-    case 2: return launch_dmma<2>(d_ops, nops, p, p_pad, st);
-    case 4: return launch_dmma<4>(d_ops, nops, p, p_pad, st);
-    case 8: return launch_dmma<8>(d_ops, nops, p, p_pad, st);
+    case 1: return launch_dmma<1>(d_ops, nops, p, p_pad, PT, st);
+    case 2: return launch_dmma<2>(d_ops, nops, p, p_pad, PT, st);
+    case 4: return launch_dmma<4>(d_ops, nops, p, p_pad, PT, st);
+    case 8: return launch_dmma<8>(d_ops, nops, p, p_pad, PT, st);
     default: return (int)cudaErrorNotSupported;
   }
 }

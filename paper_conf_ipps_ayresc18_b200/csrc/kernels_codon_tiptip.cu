@@ -1,4 +1,4 @@
-// K3-TT: 61-state codon operations whose two children are tips (fp32).
+// K3-TT: 61-state codon operations whose two children are tips (fp32, fp64).
 //
 // Eq. (1) (§II-A) with one-hot children is a gather, not a
 // contraction: sum_x P1[z][x] [x = s1] = P1[z][s1], so
@@ -41,11 +41,48 @@ __device__ inline int frexp_e_tt(float m) {
   frexpf(m, &e);
   return e;
 }
+__device__ inline int frexp_e_tt(double m) {
+  const unsigned long long b = (unsigned long long)__double_as_longlong(m);
+  const int eb = (int)((b >> 52) & 0x7ffull);
+  if (eb != 0 && eb != 0x7ff) return eb - 1022;
+  if (m == 0.0) return 0;
+  int e;
+  frexp(m, &e);
+  return e;
+}
+__device__ inline float pow2_neg_tt(float, int e) {
+  return (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23) : ldexpf(1.f, -e);
+}
+__device__ inline double pow2_neg_tt(double, int e) {
+  return (e > -1022 && e < 1022) ? __longlong_as_double((long long)(1023 - e) << 52) : ldexp(1.0, -e);
+}
 
-template <int C>
+// Four consecutive states of one row (16 bytes fp32, 32 bytes fp64).
+template <typename T> struct Q4;
+template <> struct Q4<float> {
+  float v[4];
+  __device__ void ld(const float *p) {
+    const float4 x = __ldg(reinterpret_cast<const float4 *>(p));
+    v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+  }
+  __device__ void st(float *p) const { *reinterpret_cast<float4 *>(p) = make_float4(v[0], v[1], v[2], v[3]); }
+};
+template <> struct Q4<double> {
+  double v[4];
+  __device__ void ld(const double *p) {
+    const double2 a = __ldg(reinterpret_cast<const double2 *>(p)), b = __ldg(reinterpret_cast<const double2 *>(p) + 1);
+    v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+  }
+  __device__ void st(double *p) const {
+    reinterpret_cast<double2 *>(p)[0] = make_double2(v[0], v[1]);
+    reinterpret_cast<double2 *>(p)[1] = make_double2(v[2], v[3]);
+  }
+};
+
+template <typename T, int C>
 __global__ void __launch_bounds__(kThrTT)
 k_partials_codon_tiptip(const DevOp *__restrict__ ops, int nchunks, int total, int p_pad,
-                        const float *__restrict__ PT) {
+                        const T *__restrict__ PT) {
   asm volatile("griddepcontrol.wait;" ::: "memory");  // K1 / host uploads precede this launch
   asm volatile("griddepcontrol.launch_dependents;" :::);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -58,9 +95,9 @@ k_partials_codon_tiptip(const DevOp *__restrict__ ops, int nchunks, int total, i
     if (p0 >= p) continue;  // a shorter pattern range of a partitioned call: not this op's rows
     const uint8_t *s1g = static_cast<const uint8_t *>(op.in1);
     const uint8_t *s2g = static_cast<const uint8_t *>(op.in2);
-    const float *T1 = PT + (size_t)op.mat1 * kMat;
-    const float *T2 = PT + (size_t)op.mat2 * kMat;
-    float *out = static_cast<float *>(op.out);
+    const T *T1 = PT + (size_t)op.mat1 * kMat;
+    const T *T2 = PT + (size_t)op.mat2 * kMat;
+    T *out = static_cast<T *>(op.out);
 #pragma unroll 2
     for (int k = warp * 2 + half; k < kChunkTT; k += 2 * (kThrTT / 32)) {
       const int pp = p0 + k;  // < p_tile: chunks are whole tiles
@@ -68,41 +105,45 @@ k_partials_codon_tiptip(const DevOp *__restrict__ ops, int nchunks, int total, i
       unsigned s1 = valid ? (unsigned)__ldg(s1g + pp) : 0u, s2 = valid ? (unsigned)__ldg(s2g + pp) : 0u;
       s1 = s1 < (unsigned)kMissing ? s1 : (unsigned)kMissing;
       s2 = s2 < (unsigned)kMissing ? s2 : (unsigned)kMissing;
-      float4 v[C];
-      float m = 0.f;
+      Q4<T> v[C];
+      T m = T(0);
 #pragma unroll
       for (int c = 0; c < C; ++c) {
-        const float4 a = __ldg(reinterpret_cast<const float4 *>(T1 + (size_t)c * 4096 + s1 * 64) + q);
-        const float4 b = __ldg(reinterpret_cast<const float4 *>(T2 + (size_t)c * 4096 + s2 * 64) + q);
-        v[c] = make_float4(a.x * b.x, a.y * b.y, a.z * b.z, a.w * b.w);
-        m = fmaxf(m, fmaxf(fmaxf(v[c].x, v[c].y), fmaxf(v[c].z, v[c].w)));
+        Q4<T> a, b;
+        a.ld(T1 + (size_t)c * 4096 + s1 * 64 + 4 * q);
+        b.ld(T2 + (size_t)c * 4096 + s2 * 64 + 4 * q);
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          v[c].v[i] = a.v[i] * b.v[i];
+          m = fmax(m, v[c].v[i]);
+        }
       }
 #pragma unroll
-      for (int o = 1; o < 16; o <<= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+      for (int o = 1; o < 16; o <<= 1) m = fmax(m, __shfl_xor_sync(0xffffffffu, m, o));
       int e = 0;
       if (op.scale_out != nullptr) e = frexp_e_tt(m);
       else if (op.scale_in != nullptr) e = valid ? __ldg(op.scale_in + pp) : 0;
-      const float f = !valid ? 0.f
-                      : (e > -126 && e < 126) ? __uint_as_float((unsigned)(127 - e) << 23)
-                                              : ldexpf(1.f, -e);
+      const T f = !valid ? T(0) : pow2_neg_tt(T(0), e);
 #pragma unroll
-      for (int c = 0; c < C; ++c)
-        reinterpret_cast<float4 *>(out + ((size_t)c * p_pad + pp) * 64)[q] =
-            make_float4(v[c].x * f, v[c].y * f, v[c].z * f, v[c].w * f);
+      for (int c = 0; c < C; ++c) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) v[c].v[i] *= f;
+        v[c].st(out + ((size_t)c * p_pad + pp) * 64 + 4 * q);
+      }
       if (valid && q == 0 && op.scale_out != nullptr) op.scale_out[pp] = e;
     }
   }
 }
 
-template <int C>
-int launch_tt(const DevOp *d_ops, int nops, int p, int p_pad, const float *PT, cudaStream_t st) {
+template <typename T, int C>
+int launch_tt(const DevOp *d_ops, int nops, int p, int p_pad, const T *PT, cudaStream_t st) {
   static int grid_dev[kMaxDevices] = {};
   int &grid_cap = grid_dev[device_slot()];
   if (grid_cap == 0) {
     int dev = 0, nsm = 148, per = 1;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_partials_codon_tiptip<C>, kThrTT, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per, k_partials_codon_tiptip<T, C>, kThrTT, 0);
     grid_cap = nsm * (per > 0 ? per : 1);
   }
   const int nchunks = (p + kChunkTT - 1) / kChunkTT;
@@ -117,22 +158,28 @@ int launch_tt(const DevOp *d_ops, int nops, int p, int p_pad, const float *PT, c
   at[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = at;
   cfg.numAttrs = 1;
-  return (int)cudaLaunchKernelEx(&cfg, k_partials_codon_tiptip<C>, d_ops, nchunks, (int)total, p_pad, PT);
+  return (int)cudaLaunchKernelEx(&cfg, k_partials_codon_tiptip<T, C>, d_ops, nchunks, (int)total, p_pad, PT);
+}
+
+template <typename T>
+int dispatch_tt(int c, const DevOp *d_ops, int nops, int p, int p_pad, const T *PT, cudaStream_t st) {
+  switch (c) {
+    case 1: return launch_tt<T, 1>(d_ops, nops, p, p_pad, PT, st);
+    case 2: return launch_tt<T, 2>(d_ops, nops, p, p_pad, PT, st);
+    case 4: return launch_tt<T, 4>(d_ops, nops, p, p_pad, PT, st);
+    case 8: return launch_tt<T, 8>(d_ops, nops, p, p_pad, PT, st);
+    default: return (int)cudaErrorNotSupported;
+  }
 }
 
 }  // namespace
 
-int launch_update_partials_codon_tiptip(int c, const DevOp *d_ops, int nops, int p, int p_pad, const float *d_PT,
-                                        void *stream) {
+int launch_update_partials_codon_tiptip(int prec, int c, const DevOp *d_ops, int nops, int p, int p_pad,
+                                        const void *d_PT, void *stream) {
   if (nops <= 0 || p <= 0) return 0;
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  switch (c) {
-    case 1: return launch_tt<1>(d_ops, nops, p, p_pad, d_PT, st);
-    case 2: return launch_tt<2>(d_ops, nops, p, p_pad, d_PT, st);
-    case 4: return launch_tt<4>(d_ops, nops, p, p_pad, d_PT, st);
-    case 8: return launch_tt<8>(d_ops, nops, p, p_pad, d_PT, st);
-    default: return (int)cudaErrorNotSupported;
-  }
+  return prec == 32 ? dispatch_tt<float>(c, d_ops, nops, p, p_pad, static_cast<const float *>(d_PT), st)
+                    : dispatch_tt<double>(c, d_ops, nops, p, p_pad, static_cast<const double *>(d_PT), st);
 }
 
 }  // namespace rrl

@@ -67,7 +67,7 @@ template <typename T>
 __global__ void __launch_bounds__(256)
 k_transition64(int s, int C, int items, const double *__restrict__ eig, const double *__restrict__ rates,
                const int32_t *__restrict__ idx, const double *__restrict__ tlen, T *__restrict__ P,
-               float *__restrict__ Plo, float *__restrict__ PT) {
+               float *__restrict__ Plo, T *__restrict__ PT) {
   // Persistent: V and V^-1 (the same for every matrix) are staged in shared
   // memory once per block, which then walks (matrix, category) items.
   extern __shared__ double sm[];
@@ -135,9 +135,11 @@ k_transition64(int s, int C, int items, const double *__restrict__ eig, const do
       const int xs[4] = {x0, x0 + 1, 32 + x0, 33 + x0};
 #pragma unroll
       for (int j = 0; j < 4; ++j)
-        if (xs[j] < s)
-          *reinterpret_cast<float4 *>(PT + off + xs[j] * 64 + z0) =
-              make_float4((float)acc[0][j], (float)acc[1][j], (float)acc[2][j], (float)acc[3][j]);
+        if (xs[j] < s) {
+          T *dst = PT + off + xs[j] * 64 + z0;
+#pragma unroll
+          for (int i = 0; i < 4; ++i) dst[i] = (T)acc[i][j];
+        }
       double rs[4];
 #pragma unroll
       for (int i = 0; i < 4; ++i) {
@@ -145,26 +147,29 @@ k_transition64(int s, int C, int items, const double *__restrict__ eig, const do
 #pragma unroll
         for (int o = 1; o < 16; o <<= 1) rs[i] += __shfl_xor_sync(0xffffffffu, rs[i], o);
       }
-      if ((tid & 15) == 0)
-        *reinterpret_cast<float4 *>(PT + off + kS61Row * 64 + z0) =
-            make_float4((float)rs[0], (float)rs[1], (float)rs[2], (float)rs[3]);
+      if ((tid & 15) == 0) {
+        T *dst = PT + off + kS61Row * 64 + z0;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) dst[i] = (T)rs[i];
+      }
     }
   }
 }
 
-// P^T of one stored fp32 codon matrix set (rrl_set_transition_matrix): same
-// layout and row-61 sums as K1 writes (sums in fp64 of the stored fp32 values).
-__global__ void k_codon_pt(const float *__restrict__ P, float *__restrict__ PT, int C) {
+// P^T of one stored codon matrix set (rrl_set_transition_matrix): same layout
+// and row-61 sums as K1 writes (sums in fp64 of the stored values).
+template <typename T>
+__global__ void k_codon_pt(const T *__restrict__ P, T *__restrict__ PT, int C) {
   const int c = blockIdx.x, z = threadIdx.x;  // 64 threads
-  const float *row = P + ((size_t)c * 64 + z) * 64;
-  float *pt = PT + (size_t)c * 64 * 64;
+  const T *row = P + ((size_t)c * 64 + z) * 64;
+  T *pt = PT + (size_t)c * 64 * 64;
   double sum = 0.0;
   for (int x = 0; x < 64; ++x) {
-    const float v = x < kS61Row ? row[x] : 0.f;
+    const T v = x < kS61Row ? row[x] : T(0);
     sum += (double)v;
     if (x != kS61Row) pt[x * 64 + z] = v;
   }
-  pt[kS61Row * 64 + z] = (float)sum;
+  pt[kS61Row * 64 + z] = (T)sum;
 }
 
 __global__ void k_split_tf32(const float *__restrict__ x, float *__restrict__ lo, size_t n) {
@@ -352,7 +357,8 @@ int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *
                                                        static_cast<float *>(d_PT));
     else
       k_transition64<double><<<grid, 256, smem64, st>>>(s, c, items, d_eig, d_rates, d_idx, d_t,
-                                                        static_cast<double *>(d_P), nullptr, nullptr);
+                                                        static_cast<double *>(d_P), nullptr,
+                                                        static_cast<double *>(d_PT));
     return (int)cudaGetLastError();
   }
   const size_t smem = sizeof(double) * (2 * s * s + s);
@@ -414,8 +420,12 @@ int launch_edge_lnl(int prec, int s, int s_pad, int c, const void *par, const vo
   return (int)cudaGetLastError();
 }
 
-int launch_codon_pt(const float *P, float *PT, int c, void *stream) {
-  k_codon_pt<<<c, 64, 0, static_cast<cudaStream_t>(stream)>>>(P, PT, c);
+int launch_codon_pt(int prec, const void *P, void *PT, int c, void *stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (prec == 32)
+    k_codon_pt<float><<<c, 64, 0, st>>>(static_cast<const float *>(P), static_cast<float *>(PT), c);
+  else
+    k_codon_pt<double><<<c, 64, 0, st>>>(static_cast<const double *>(P), static_cast<double *>(PT), c);
   return (int)cudaGetLastError();
 }
 

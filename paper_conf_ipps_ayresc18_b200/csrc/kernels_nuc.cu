@@ -41,16 +41,21 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr int kInline = 8;
-// Latency path: 4 resident 256-thread CTAs per SM (<= 64 registers), so the
-// next level set's CTAs (2 per SM at configs[1]) are co-resident with the
-// current set's under programmatic dependent launch and run their prologue
-// (descriptors, tip states, P rows) before griddepcontrol.wait instead of
-// after the previous grid's exit.
+// Latency path: the transition tables live in shared memory (staged before
+// griddepcontrol.wait when K1 is not the immediate predecessor) instead of 32
+// registers per thread, and the CTA is held to 5 resident per SM (48
+// registers, no spills), so the next level set's CTAs (2.1 per SM at
+// configs[1]) are resident beside the current set's under programmatic
+// dependent launch and finish their whole prologue before its wait.
+// Measured on configs[1] (updatePartials per pass, fp32): rows in registers,
+// 80 registers 0.173 ms; tables in shared memory at 3 / 4 / 5 / 6 CTAs per SM
+// 0.163 / 0.178 (spills) / 0.145 / 0.169 ms.  fp64 (tables in shared memory
+// already) keeps 3 CTAs per SM: at 5 it spills and is no faster (0.214 ms).
 #ifndef RRL_LAT_MINB
-#define RRL_LAT_MINB 3
+#define RRL_LAT_MINB 5
 #endif
 #ifndef RRL_LAT_PSMEM
-#define RRL_LAT_PSMEM 0
+#define RRL_LAT_PSMEM 1
 #endif
 constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 constexpr int kChunkItems = 512;  // items (pattern x category) per bulk chunk
@@ -220,7 +225,7 @@ __device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
 // level set passed its own wait).  Only the previous level set's partials and
 // exponents must wait.
 template <typename T, int C, int U>
-__global__ void __launch_bounds__(kThreads, kLatencyMinBlocks)
+__global__ void __launch_bounds__(kThreads, sizeof(T) == 4 ? kLatencyMinBlocks : 3)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int early) {
   const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;

@@ -77,18 +77,19 @@ int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_o
                                      int p_pad, const void *tmap_partials, const void *tmap_P,
                                      const void *tmap_Plo, void *stream);
 // fp64 codon operations on the FP64 tensor cores (mma.sync m8n8k4 f64), c in {1, 2, 4, 8}.
-int launch_update_partials_codon_dmma(int c, const DevOp *d_ops, int nops, int p, int p_pad, void *stream);
+int launch_update_partials_codon_dmma(int c, const DevOp *d_ops, int nops, int p, int p_pad, const void *d_PT,
+                                      void *stream);
 // *flag = 1 if any of `bytes` (multiple of 16) uint8 tip codes exceeds s, else 0.
 int launch_check_states(const uint8_t *d, size_t bytes, int s, unsigned *flag, void *stream);
 int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *d_eig,
                                const double *d_rates, const int32_t *d_idx, const double *d_t,
                                int count, void *d_P, void *d_Plo, void *d_PT, void *stream);
-// P^T of one fp32 codon matrix set [c][64][64] (row 61 = row sums), as K1 writes it.
-int launch_codon_pt(const float *P, float *PT, int c, void *stream);
-// 61-state fp32 operations whose two children are tips (first level set):
-// dest[c][p][z] = P1[c][z][s1] P2[c][z][s2] from the P^T slab, rescaled.
-int launch_update_partials_codon_tiptip(int c, const DevOp *d_ops, int nops, int p, int p_pad, const float *d_PT,
-                                        void *stream);
+// P^T of one codon matrix set [c][64][64] (row 61 = row sums), as K1 writes it.
+int launch_codon_pt(int prec, const void *P, void *PT, int c, void *stream);
+// 61-state operations whose two children are tips (first level set), fp32 or
+// fp64: dest[c][p][z] = P1[c][z][s1] P2[c][z][s2] from the P^T slab, rescaled.
+int launch_update_partials_codon_tiptip(int prec, int c, const DevOp *d_ops, int nops, int p, int p_pad,
+                                        const void *d_PT, void *stream);
 int launch_accumulate_scale(const int32_t *d_scale, int p_pad, const int32_t *d_idx, int count,
                             int32_t *d_cum, int p, void *stream);
 int launch_root_lnl(int prec, int s, int s_pad, int c, const void *root, const double *d_w,
