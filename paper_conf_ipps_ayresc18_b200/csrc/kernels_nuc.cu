@@ -58,6 +58,10 @@ constexpr int kInline = 8;
 #define RRL_LAT_PSMEM 1
 #endif
 constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
+#ifndef RRL_LAT_THREADS
+#define RRL_LAT_THREADS 256
+#endif
+constexpr int kLatThreads = RRL_LAT_THREADS;  // latency-path CTA size
 constexpr int kChunkItems = 512;  // items (pattern x category) per bulk chunk
 constexpr int kPTab = 36;         // per (branch, cat): 16 rows P[z][x] + 5 columns x 4
 
@@ -225,11 +229,11 @@ __device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
 // level set passed its own wait).  Only the previous level set's partials and
 // exponents must wait.
 template <typename T, int C, int U>
-__global__ void __launch_bounds__(kThreads, sizeof(T) == 4 ? kLatencyMinBlocks : 3)
+__global__ void __launch_bounds__(kLatThreads, sizeof(T) == 4 ? kLatencyMinBlocks : 3)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int early) {
   const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
-  const int cat = threadIdx.x % C;  // kThreads is a multiple of C
+  const int cat = threadIdx.x % C;  // kLatThreads is a multiple of C
   const T *__restrict__ P1g = static_cast<const T *>(op.P1) + cat * 16;
   const T *__restrict__ P2g = static_cast<const T *>(op.P2) + cat * 16;
   const T *__restrict__ L1g = static_cast<const T *>(op.in1);
@@ -261,7 +265,7 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
   if (early & 1) {
 #pragma unroll
     for (int j = 0; j < U; ++j) {
-      const unsigned item = (unsigned)blockIdx.x * (kThreads * U) + threadIdx.x + j * kThreads;
+      const unsigned item = (unsigned)blockIdx.x * (kLatThreads * U) + threadIdx.x + j * kLatThreads;
       const bool valid = item < nitems && (int)blockIdx.x < nchunks;
       s1p[j] = (tip1 && valid) ? (unsigned)__ldg(S1g + item / C) : 4u;
       s2p[j] = (tip2 && valid) ? (unsigned)__ldg(S2g + item / C) : 4u;
@@ -282,13 +286,13 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
   if (!(early & 2)) load_rows();
   for (int chunk = blockIdx.x; chunk < nchunks; chunk += gridDim.x) {
     const bool pre = (early & 1) && chunk == (int)blockIdx.x;
-    const unsigned base = (unsigned)chunk * (kThreads * U) + threadIdx.x;
+    const unsigned base = (unsigned)chunk * (kLatThreads * U) + threadIdx.x;
     T L1[U][4], L2[U][4];
     unsigned s1[U], s2[U];
     int ca[U], cb[U];
 #pragma unroll
     for (int j = 0; j < U; ++j) {  // ---- all reads of this thread in flight together
-      const unsigned item = base + j * kThreads;
+      const unsigned item = base + j * kLatThreads;
       const bool valid = item < nitems;
       const unsigned pat = item / C;
       if (tip1) {
@@ -318,7 +322,7 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
     }
 #pragma unroll
     for (int j = 0; j < U; ++j) {  // ---- compute + store
-      const unsigned item = base + j * kThreads;
+      const unsigned item = base + j * kLatThreads;
       const bool valid = item < nitems;
       const unsigned pat = item / C;
       T v1[4], v2[4], r[4];
@@ -840,7 +844,7 @@ template <typename T, int C, int U>
 int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int gx_cap, int early,
                      cudaStream_t st) {
   const long long items = (long long)p * C;
-  const int nchunks = (int)((items + kThreads * U - 1) / (kThreads * U));
+  const int nchunks = (int)((items + kLatThreads * U - 1) / (kLatThreads * U));
   int gx = gx_cap / nops;
   if (gx > nchunks) gx = nchunks;
   if (gx < 1) gx = 1;
@@ -854,7 +858,7 @@ int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, in
     if (ny <= kInline && h_ops == nullptr) pack.n = kInline + 1;  // force pointer path
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3(gx, ny);
-    cfg.blockDim = dim3(kThreads);
+    cfg.blockDim = dim3(kLatThreads);
     cfg.stream = st;
     cudaLaunchAttribute at[1];
     at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
@@ -878,7 +882,7 @@ int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int 
   int &resident = resident_dev[device_slot()];
   if (resident <= 0) {
     int per_sm = 1, dev = 0, nsm = 148;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, 1>, kThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, 1>, kLatThreads, 0);
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     resident = (per_sm > 0 ? per_sm : 1) * nsm;
