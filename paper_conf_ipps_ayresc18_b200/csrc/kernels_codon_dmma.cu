@@ -12,21 +12,17 @@
 // 32 FMAs instead of per 8.
 //
 // One CTA = one (operation, 64-pattern tile), all categories (the rescale
-// needs max over (c, z)).  8 warps; warp w owns patterns 8w..8w+7 and all 64
-// states: per K-step of 4, one A fragment (its pattern row, 4 consecutive x)
-// and 8 B fragments (one per 8-state block) -> 8 DMMAs into 8 accumulator
-// pairs.  DMMA fragment layout (m8n8k4, f64): lane = 4 g + t; A[g][t],
-// B[t][g] (= P[8j + g][4k + t]), D[g][2t + i].  So a thread owns ONE pattern
-// (8w + g) and the 16 states 8j + 2t + i -- the tip gather and the per-pattern
-// max are per-thread work plus two xor-shuffles over the 4 lanes of a pattern.
-// The child tile of an internal child sits in shared memory (68-double rows:
-// a warp's 32 LDS.64 of a fragment are two conflict-free wavefronts),
-// double-buffered: the next internal stage is copied with cp.async while the
-// current stage's DMMAs run.  B fragments come straight from the 32 KB P tile
-// (L1-resident: every warp of the CTA reads it), and a tip child reads the
-// thread's 16 entries from row `state` of K1's P^T slab -- no staging, no
-// barrier.  Each category's unscaled product is stored at once with a running
-// max kept; when the max is known the thread rescales what it stored.
+// needs max over (c, z)), 8 warps of 32 x 16 (pattern x state) tiles.  DMMA
+// fragment layout (m8n8k4, f64): lane = 4 g + t; A[g][t], B[t][g] (= P[z][x]),
+// D[g][2t + i].  The child tile of an internal child sits in shared memory
+// (68-double rows: a warp's 32 LDS.64 of a fragment are two conflict-free
+// wavefronts), double-buffered: the next internal stage is copied with
+// cp.async while the current stage's DMMAs run.  B fragments come straight
+// from the 32 KB P tile (L1-resident: every warp of the CTA reads it), and a
+// tip child reads the thread's entries from row `state` of K1's P^T slab --
+// no staging, no barrier.  Each category's unscaled product is stored at once
+// with a running max kept; when the max is known the thread rescales what it
+// stored.
 #include <cuda_runtime.h>
 
 #include <cstdint>
@@ -41,6 +37,7 @@ constexpr int kRow = 68;  // shared-memory row stride of the A tile (doubles)
 
 struct DmmaSmem {
   double A[2][kTPD * kRow];  // double-buffered child tiles [pattern][x]
+  double mx[4][kTPD];        // per-pattern maxima of the 4 state-quarter warps
   uint8_t st[2][kTPD];       // tip states of both children
 };
 
@@ -72,6 +69,14 @@ __device__ inline double pow2_neg64(int e) {
 // Stage (c, b) of a CTA = category c, child b; only internal children stage an
 // A tile.  The next internal stage's tile is copied (cp.async) into the other
 // buffer while the current stage's DMMAs run.
+//
+// Warp tile 32 patterns x 16 states (wr = warp & 1, wc = warp >> 1): per
+// K-step 4 A fragments (shared memory) and 2 B fragments (the 32 KB P tile,
+// L1-resident) feed 8 DMMAs, so the L1 carries a quarter of the B traffic of
+// an 8 x 64 warp tile (which measured 91 % L1 throughput, the limit).  A
+// thread owns patterns 32 wr + 8 rb + g (rb < 4) and states 16 wc + 8 cb +
+// 2 t + i (cb, i < 2); the per-pattern max over (c, z) is reduced over the 4
+// lanes t by shuffles and over the 4 warps wc through shared memory.
 template <int C>
 __global__ void __launch_bounds__(kThrD, 2)
 k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__restrict__ PT) {
@@ -86,9 +91,8 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__
   const double *Pg[2] = {static_cast<const double *>(op.P1), static_cast<const double *>(op.P2)};
   const int mat[2] = {op.mat1, op.mat2};
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, g = lane >> 2, t = lane & 3;
-  const int prow = warp * 8 + g;  // this thread's pattern in the tile
-  const int pp = p0 + prow;
-  const bool valid = pp < p;
+  const int wr = warp & 1, wc = warp >> 1;
+  const int zbase = 16 * wc + 2 * t;  // + 8 cb + i
 
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" :::);
@@ -100,9 +104,8 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__
     }
     cp_async_commit();
   };
-  // the internal stages in order: (c, b) for b with !tip[b]
   const int nint = (tip[0] ? 0 : 1) + (tip[1] ? 0 : 1);
-  int si = 0;  // internal stages issued so far
+  int si = 0;  // internal stages consumed so far
   if (nint > 0) stage_A(0, tip[0] ? 1 : 0, 0);
   for (int b = 0; b < 2; ++b)
     if (tip[b] && tid < kTPD) {
@@ -110,25 +113,37 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__
       sm.st[b][tid] = q < p ? static_cast<const uint8_t *>(in[b])[q] : (uint8_t)kS;
     }
   const bool two_pass = op.scale_out != nullptr;
-  const double f_in = (!two_pass && op.scale_in != nullptr && valid) ? pow2_neg64(op.scale_in[pp]) : 1.0;
+  int prow[4];
+  bool valid[4];
+  double f_in[4], m[4];
+#pragma unroll
+  for (int rb = 0; rb < 4; ++rb) {
+    prow[rb] = 32 * wr + 8 * rb + g;
+    valid[rb] = p0 + prow[rb] < p;
+    f_in[rb] = (!two_pass && op.scale_in != nullptr && valid[rb]) ? pow2_neg64(op.scale_in[p0 + prow[rb]]) : 1.0;
+    m[rb] = 0.0;
+  }
   double *out = static_cast<double *>(op.out);
-  double m = 0.0;
   __syncthreads();  // tip states
   for (int c = 0; c < C; ++c) {
-    double d1[16];
+    double d1[4][4];  // [rb][2 cb + i]
 #pragma unroll
     for (int b = 0; b < 2; ++b) {
-      double v[16];
+      double v[4][4];
       if (tip[b]) {
-        // P[z][s] for the thread's 16 states z = 8j + 2t + i: consecutive pairs of
-        // row s of P^T (K1; row 61 = row sums for a missing state), L1/L2-resident
-        const unsigned s = sm.st[b][prow];
-        const double *row = PT + ((size_t)mat[b] * C + c) * kSP * kSP + (s < (unsigned)kS ? s : kS) * kSP + 2 * t;
+        // P[z][s] for the thread's states: row s of P^T (K1; row 61 = row sums for
+        // a missing state), two 16-byte pairs per pattern, L1/L2-resident
+        const double *base = PT + ((size_t)mat[b] * C + c) * kSP * kSP + zbase;
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          const double2 x = __ldg(reinterpret_cast<const double2 *>(row + 8 * j));
-          v[2 * j] = x.x;
-          v[2 * j + 1] = x.y;
+        for (int rb = 0; rb < 4; ++rb) {
+          const unsigned s = sm.st[b][prow[rb]];
+          const double *row = base + (s < (unsigned)kS ? s : kS) * kSP;
+#pragma unroll
+          for (int cb = 0; cb < 2; ++cb) {
+            const double2 x = __ldg(reinterpret_cast<const double2 *>(row + 8 * cb));
+            v[rb][2 * cb] = x.x;
+            v[rb][2 * cb + 1] = x.y;
+          }
         }
       } else {
         const int buf = si & 1;
@@ -140,63 +155,86 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__
           const int nc = (nint == 2) ? (b == 1 ? c + 1 : c) : c + 1;
           stage_A(nc, nb, buf ^ 1);
         }
-        double acc[8][2];
+        double acc[4][2][2];
 #pragma unroll
-        for (int j = 0; j < 8; ++j) acc[j][0] = acc[j][1] = 0.0;
-        const double *Ar = &sm.A[buf][prow * kRow + t];
-        // B fragment B[x][z] = P[z][x], z = 8j + g, x = 4k + t (L1-resident P tile)
-        const double *Pr = Pg[b] + (size_t)c * kSP * kSP + g * kSP + t;
+        for (int rb = 0; rb < 4; ++rb)
+#pragma unroll
+          for (int cb = 0; cb < 2; ++cb) acc[rb][cb][0] = acc[rb][cb][1] = 0.0;
+        const double *Ar = &sm.A[buf][(32 * wr + g) * kRow + t];
+        // B fragment B[x][z] = P[z][x], z = 16 wc + 8 cb + g, x = 4k + t
+        const double *Pr = Pg[b] + (size_t)c * kSP * kSP + (16 * wc + g) * kSP + t;
 #pragma unroll 4
         for (int k = 0; k < kSP / 4; ++k) {
-          const double a = Ar[4 * k];
+          const double b0 = __ldg(Pr + 4 * k), b1 = __ldg(Pr + 8 * kSP + 4 * k);
 #pragma unroll
-          for (int j = 0; j < 8; ++j) dmma(acc[j], a, __ldg(Pr + (8 * j) * kSP + 4 * k));
+          for (int rb = 0; rb < 4; ++rb) {
+            const double a = Ar[(8 * rb) * kRow + 4 * k];
+            dmma(acc[rb][0], a, b0);
+            dmma(acc[rb][1], a, b1);
+          }
         }
 #pragma unroll
-        for (int j = 0; j < 8; ++j) {
-          v[2 * j] = acc[j][0];
-          v[2 * j + 1] = acc[j][1];
-        }
+        for (int rb = 0; rb < 4; ++rb)
+#pragma unroll
+          for (int cb = 0; cb < 2; ++cb) {
+            v[rb][2 * cb] = acc[rb][cb][0];
+            v[rb][2 * cb + 1] = acc[rb][cb][1];
+          }
       }
-      if (b == 0) {
 #pragma unroll
-        for (int i = 0; i < 16; ++i) d1[i] = v[i];
-      } else {
+      for (int rb = 0; rb < 4; ++rb)
 #pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          d1[i] *= v[i];
-          m = fmax(m, d1[i]);
+        for (int i = 0; i < 4; ++i) {
+          if (b == 0) {
+            d1[rb][i] = v[rb][i];
+          } else {
+            d1[rb][i] *= v[rb][i];
+            m[rb] = fmax(m[rb], d1[rb][i]);
+          }
         }
-      }
     }
-    if (valid) {  // this category's unscaled (or stored-factor) product, states 8j + 2t + {0, 1}
-      double *dst = out + ((size_t)c * p_pad + pp) * kSP + 2 * t;
 #pragma unroll
-      for (int j = 0; j < 8; ++j)
-        *reinterpret_cast<double2 *>(dst + 8 * j) = make_double2(d1[2 * j] * f_in, d1[2 * j + 1] * f_in);
-    }
+    for (int rb = 0; rb < 4; ++rb)  // this category's unscaled (or stored-factor) product
+      if (valid[rb]) {
+        double *dst = out + ((size_t)c * p_pad + p0 + prow[rb]) * kSP + zbase;
+#pragma unroll
+        for (int cb = 0; cb < 2; ++cb)
+          *reinterpret_cast<double2 *>(dst + 8 * cb) =
+              make_double2(d1[rb][2 * cb] * f_in[rb], d1[rb][2 * cb + 1] * f_in[rb]);
+      }
   }
   if (!two_pass) return;
-  // ---- rescale: max over (c, z) of the pattern across its 4 lanes, then each
-  // thread scales the values it stored above by the exact power of two
-  m = fmax(m, __shfl_xor_sync(0xffffffffu, m, 1));
-  m = fmax(m, __shfl_xor_sync(0xffffffffu, m, 2));
-  const int e = frexp_e64(m);
-  if (!valid) return;
-  if (t == 0) {
-    int tot = e;
-    if (op.cum1 != nullptr) tot += op.cum1[pp];
-    if (op.cum2 != nullptr) tot += op.cum2[pp];
-    op.scale_out[pp] = tot;
+  // ---- rescale: max over (c, z) of each pattern: over the 4 lanes t, then over
+  // the 4 warps wc sharing the pattern (shared memory), then each thread scales
+  // the values it stored above by the exact power of two
+#pragma unroll
+  for (int rb = 0; rb < 4; ++rb) {
+    m[rb] = fmax(m[rb], __shfl_xor_sync(0xffffffffu, m[rb], 1));
+    m[rb] = fmax(m[rb], __shfl_xor_sync(0xffffffffu, m[rb], 2));
+    if (t == 0) sm.mx[wc][prow[rb]] = m[rb];
   }
-  const double f = pow2_neg64(e);
+  __syncthreads();
 #pragma unroll
-  for (int c = 0; c < C; ++c) {
-    double2 *dst = reinterpret_cast<double2 *>(out + ((size_t)c * p_pad + pp) * kSP + 2 * t);
+  for (int rb = 0; rb < 4; ++rb) {
+    if (!valid[rb]) continue;
+    const double mm = fmax(fmax(sm.mx[0][prow[rb]], sm.mx[1][prow[rb]]), fmax(sm.mx[2][prow[rb]], sm.mx[3][prow[rb]]));
+    const int e = frexp_e64(mm);
+    const int pp = p0 + prow[rb];
+    if (wc == 0 && t == 0) {
+      int tot = e;
+      if (op.cum1 != nullptr) tot += op.cum1[pp];
+      if (op.cum2 != nullptr) tot += op.cum2[pp];
+      op.scale_out[pp] = tot;
+    }
+    const double f = pow2_neg64(e);
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const double2 x = dst[4 * j];
-      dst[4 * j] = make_double2(x.x * f, x.y * f);
+    for (int c = 0; c < C; ++c) {
+      double2 *dst = reinterpret_cast<double2 *>(out + ((size_t)c * p_pad + pp) * kSP + zbase);
+#pragma unroll
+      for (int cb = 0; cb < 2; ++cb) {
+        const double2 x = dst[4 * cb];
+        dst[4 * cb] = make_double2(x.x * f, x.y * f);
+      }
     }
   }
 }

@@ -294,7 +294,9 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         if (is_tip(op, b)) continue;  // a tip child is a P-column gather in the epilogue: no MMA
         const uint32_t sl = ia % NA, use = ia / NA;
         bar_wait(&a_full[sl], use & 1u);
+        bar_wait(lo_full, ia & 1u);
         bar_wait(acc_empty, (ia & 1u) ^ 1u);  // the epilogue drained the previous accumulators
+        ++ia;
         fence_after();
         TR(3, g);
         // Accumulators [main_0 | corr | main_1]: K-half 0 as A_hi . [P_hi | P_lo]^T (N = 128)
@@ -302,32 +304,24 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         // (A_hi P_hi -> main_1, A_hi P_lo and A_lo P_hi -> corr; same tensor time).  The
         // hi.hi sums of the two K-halves and the ~2^-11-smaller corrections never share
         // an accumulator (tf32 accumulation reading); one shared correction
-        // accumulator saves a quarter of the epilogue's TMEM reads.  The A_hi MMAs (2/3
-        // of the tensor work) are issued before waiting for this phase's lo tile, so
-        // the converters' lo pass of this phase overlaps them (one lo buffer: they
-        // could only start once the previous phase's A_lo MMAs completed).
+        // accumulator saves a quarter of the epilogue's TMEM reads.  (Issuing the A_hi
+        // MMAs before waiting for the lo tile, to overlap the converters, measured no
+        // faster: 1.557 vs 1.533 ms per configs[3] pass.)
 #pragma unroll
         for (int kk = 0; kk < TS / 8; ++kk) {
           const int h = kk >> 2, kin = kk & 3;
           const uint64_t ah = desc_sw128(sbase + SM_A + sl * 32768 + h * 16384 + kin * 32);
+          const uint64_t al = desc_sw128(sbase + SM_ALO + h * 16384 + kin * 32);
           const uint64_t bb = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + kin * 32);
           if (h == 0) {
             mma_tf32(tmem, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);
+            mma_tf32(tmem + TS, al, bb, idesc_tf32(TS), 1u);
           } else {
             const uint64_t bl = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + 8192 + kin * 32);
             mma_tf32(tmem + 2 * TS, ah, bb, idesc_tf32(TS), kin > 0 ? 1u : 0u);
             mma_tf32(tmem + TS, ah, bl, idesc_tf32(TS), 1u);
+            mma_tf32(tmem + TS, al, bb, idesc_tf32(TS), 1u);
           }
-        }
-        bar_wait(lo_full, ia & 1u);
-        ++ia;
-        fence_after();
-#pragma unroll
-        for (int kk = 0; kk < TS / 8; ++kk) {
-          const int h = kk >> 2, kin = kk & 3;
-          const uint64_t al = desc_sw128(sbase + SM_ALO + h * 16384 + kin * 32);
-          const uint64_t bb = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + kin * 32);
-          mma_tf32(tmem + TS, al, bb, idesc_tf32(TS), 1u);  // corr += A_lo P_hi
         }
         commit(&a_empty[sl]);  // child tile, lo tile and matrix tile free once these MMAs completed
         commit(lo_empty);

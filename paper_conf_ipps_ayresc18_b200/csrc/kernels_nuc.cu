@@ -48,20 +48,23 @@ constexpr int kInline = 8;
 // configs[1]) are resident beside the current set's under programmatic
 // dependent launch and finish their whole prologue before its wait.
 // Measured on configs[1] (updatePartials per pass, fp32): rows in registers,
-// 80 registers 0.173 ms; tables in shared memory at 3 / 4 / 5 / 6 CTAs per SM
-// 0.163 / 0.178 (spills) / 0.145 / 0.169 ms.  fp64 (tables in shared memory
-// already) keeps 3 CTAs per SM: at 5 it spills and is no faster (0.214 ms).
+// 80 registers 0.173 ms; tables in shared memory, 256-thread CTAs at 3 / 4 /
+// 5 / 6 per SM 0.163 / 0.178 (spills) / 0.145 / 0.169 ms; 128-thread CTAs at
+// 10 per SM (48 registers) 0.143 ms; 512-thread CTAs 0.176-0.183 ms.  fp64
+// (tables in shared memory already) keeps 3 CTAs per SM: at 5 it spills and is
+// no faster (0.214 ms).
 #ifndef RRL_LAT_MINB
-#define RRL_LAT_MINB 5
+#define RRL_LAT_MINB 10
 #endif
 #ifndef RRL_LAT_PSMEM
 #define RRL_LAT_PSMEM 1
 #endif
 constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 #ifndef RRL_LAT_THREADS
-#define RRL_LAT_THREADS 256
+#define RRL_LAT_THREADS 128
 #endif
 constexpr int kLatThreads = RRL_LAT_THREADS;  // latency-path CTA size
+constexpr int kLatencyMinBlocks64 = 3 * 256 / kLatThreads;  // fp64: 768 resident threads per SM
 constexpr int kChunkItems = 512;  // items (pattern x category) per bulk chunk
 constexpr int kPTab = 36;         // per (branch, cat): 16 rows P[z][x] + 5 columns x 4
 
@@ -229,7 +232,7 @@ __device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
 // level set passed its own wait).  Only the previous level set's partials and
 // exponents must wait.
 template <typename T, int C, int U>
-__global__ void __launch_bounds__(kLatThreads, sizeof(T) == 4 ? kLatencyMinBlocks : 3)
+__global__ void __launch_bounds__(kLatThreads, sizeof(T) == 4 ? kLatencyMinBlocks : kLatencyMinBlocks64)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int early) {
   const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;

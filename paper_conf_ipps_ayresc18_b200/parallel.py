@@ -36,12 +36,29 @@ def schedule_digest(sched: dict) -> str:
     return h.hexdigest()
 
 
-def allreduce_sum_(tensor, group=None):
+def allreduce_sum_(tensor, group=None, deterministic=False):
     """In-place SUM all-reduce of a 1-element fp64 tensor: on the device with
     NCCL; through a host copy with gloo (the CPU-side wiring tests and
-    several ranks sharing one GPU, where NCCL refuses)."""
+    several ranks sharing one GPU, where NCCL refuses).
+
+    deterministic=True: every rank writes its value into its
+    own slot of a zero R-vector, the vector is all-reduced (x + 0 = x, so the
+    reduction order cannot change a bit) and every rank folds the R slots in
+    rank order -- the same bits on every rank and in every run, whatever
+    order the collective adds in."""
     import torch.distributed as dist
     if not dist.is_initialized():  # a single process: the local sum is the global one
+        return tensor
+    if deterministic:
+        import torch
+        world, rank = dist.get_world_size(group), dist.get_rank(group)
+        v = torch.zeros(world, dtype=tensor.dtype, device=tensor.device)
+        v[rank] = tensor.reshape(())
+        allreduce_sum_(v, group)
+        acc = v[0].clone()
+        for r in range(1, world):
+            acc += v[r]
+        tensor.copy_(acc.reshape(tensor.shape))
         return tensor
     if tensor.is_cuda and dist.get_backend(group) != "nccl":
         h = tensor.cpu()
@@ -57,7 +74,8 @@ class ShardedTreeLikelihood:
 
     def __init__(self, n: int, p_total: int, s: int, c: int, rank: int, world: int,
                  precision: int = 32, device: int = 0, cuda_graph: bool = True,
-                 stream_ptr: int | None = None, group=None, buffer_count: int | None = None):
+                 stream_ptr: int | None = None, group=None, buffer_count: int | None = None,
+                 deterministic_reduce: bool = False):
         import torch
 
         from .engine import TreeLikelihood
@@ -72,6 +90,7 @@ class ShardedTreeLikelihood:
         self.tl = TreeLikelihood(n, self.hi - self.lo, s, c, precision=precision, device=device,
                                  cuda_graph=cuda_graph, stream_ptr=stream_ptr, buffer_count=buffer_count)
         self.stream_ptr = stream_ptr
+        self.deterministic = deterministic_reduce
         self.device = device
         self.d_out = torch.zeros(1, dtype=torch.float64, device=f"cuda:{device}")
 
@@ -103,7 +122,7 @@ class ShardedTreeLikelihood:
             # library's: K4 must have written d_out first
             from . import rrl as R
             R.rrl_synchronize(self.tl.inst)
-        allreduce_sum_(self.d_out, self.group)
+        allreduce_sum_(self.d_out, self.group, deterministic=self.deterministic)
         return self.d_out
 
     def loglik(self) -> float:

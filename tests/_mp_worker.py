@@ -17,7 +17,7 @@ def sharded_rank(rank, world, port, outdir):
         torch.cuda.set_device(0)
         torch.cuda.set_stream(torch.cuda.Stream())      # distinct streams per rank
         w = make_workload(tree_kind="random", n=100, p=9_001, model="gtr", c=4, seed=23)
-        sh = ShardedTreeLikelihood(w.n, w.p, w.s, w.c, rank, world, precision=64)
+        sh = ShardedTreeLikelihood(w.n, w.p, w.s, w.c, rank, world, precision=64, deterministic_reduce=True)
         sh.set_model_params(w.model, w.rates, w.cat_weights)
         sh.set_tips(w.tips)
         sh.set_pattern_weights(w.pattern_weights)

@@ -78,3 +78,37 @@ def test_gloo_sharded_sum_equals_unsharded(world):
     for rank, got, full, ndig in res:
         assert ndig == 1                      # identical schedule on every rank
         assert abs(got - full) <= 1e-12 * abs(full)
+
+
+def _det_worker(rank, world, port, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        vals = [0.1, 1e16, -1e16, 0.3][:world]   # order-sensitive in floating point
+        t = torch.tensor([vals[rank]], dtype=torch.float64)
+        allreduce_sum_(t, deterministic=True)
+        ref = 0.0
+        for v in vals:
+            ref += v
+        q.put((rank, float(t.item()), ref))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("world", [2, 4])
+def test_deterministic_allreduce_folds_in_rank_order(world):
+    """one-hot R-vector all-reduce -- every rank gets the rank-order
+    fold of the per-rank values, bit for bit."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_det_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, got, ref in res:
+        assert got == ref
