@@ -19,6 +19,12 @@ METRICS = [
     ("sm__throughput.avg.pct_of_peak_sustained_elapsed", "sm_%"),
     ("sm__warps_active.avg.pct_of_peak_sustained_active", "warps_active_%"),
     ("smsp__inst_executed.sum", "inst"),
+    # tensor pipes: tcgen05 (hmma subpipe, UTC*MMA) and DMMA (fp64 mma.sync)
+    ("sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_active", "tensor_pipe_%"),
+    ("sm__pipe_tensor_subpipe_hmma_cycles_active.avg.pct_of_peak_sustained_active", "hmma_subpipe_%"),
+    ("sm__pipe_tensor_subpipe_dmma_cycles_active.avg.pct_of_peak_sustained_active", "dmma_subpipe_%"),
+    ("sm__pipe_tc_cycles_active.avg.pct_of_peak_sustained_active", "tc_pipe_%"),
+    ("l1tex__throughput.avg.pct_of_peak_sustained_active", "l1tex_%"),
 ]
 
 
