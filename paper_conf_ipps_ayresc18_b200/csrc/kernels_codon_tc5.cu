@@ -69,8 +69,17 @@ constexpr int kThr = 15 * 32;
 // 16 KB K-halves each), one tile of lo parts, a ring of two matrix tiles (per
 // K-half h: [P hi rows 0-63 | P lo rows 0-63], 16 KB, so one N = 128 MMA reads
 // A hi once for hi.hi and hi.lo), the output staging tile.
-constexpr int NA = 3, NB = 2;
-constexpr int SM_A = 0, SM_ALO = NA * 32768, SM_B = SM_ALO + 32768, SM_S1 = SM_B + NB * 32768;
+#ifndef RRL_TC5_NLO
+#define RRL_TC5_NLO 1
+#endif
+#ifndef RRL_TC5_NB
+#define RRL_TC5_NB 2
+#endif
+constexpr int NLO = RRL_TC5_NLO;  // lo tiles (2: the converters run under the previous phase's MMAs)
+constexpr int NB = RRL_TC5_NB;    // matrix tiles (3: a tip phase's P tile lands while the previous one is read)
+constexpr int NA = 6 - NLO - NB;  // child tiles; 6 x 32 KB of rings + the staging tile fit 227 KB
+constexpr int SM_A = 0, SM_ALO = NA * 32768, SM_B = SM_ALO + NLO * 32768, SM_S1 = SM_B + NB * 32768;
+static_assert(NA >= 1 && 2 * (NA + NB + NLO) + 2 <= 16, "ring sizes / mbarrier slots");
 constexpr int SMEM_MX = SM_S1 + TM * TS * 4;           // row maxima / scale [2][128]
 constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 16 mbarriers
 constexpr int SMEM_TMEM = SMEM_BAR + 16 * 8;
@@ -179,10 +188,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
   uint64_t *a_empty = a_full + NA;                                  // [NA] its MMAs completed
   uint64_t *b_full = a_full + 2 * NA;                               // [NB] matrix tile landed
   uint64_t *b_empty = b_full + NB;                                  // [NB] MMAs / tip gather done
-  uint64_t *lo_full = b_full + 2 * NB;                              // converters wrote the lo tile
-  uint64_t *lo_empty = lo_full + 1;                                 // its MMAs completed
-  uint64_t *acc_full = lo_full + 2;
-  uint64_t *acc_empty = lo_full + 3;
+  uint64_t *lo_full = b_full + 2 * NB;                              // [NLO] converters wrote the lo tile
+  uint64_t *lo_empty = lo_full + NLO;                               // [NLO] its MMAs completed
+  uint64_t *acc_full = lo_full + 2 * NLO;
+  uint64_t *acc_empty = acc_full + 1;
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(sm + SMEM_TMEM);
   float *S1 = reinterpret_cast<float *>(sm + SM_S1);
   float *mx = reinterpret_cast<float *>(sm + SMEM_MX);
@@ -204,8 +213,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       bar_init(&b_full[i], 1);
       bar_init(&b_empty[i], 1);
     }
-    bar_init(lo_full, kConvThr / 32);
-    bar_init(lo_empty, 1);
+    for (int i = 0; i < NLO; ++i) {
+      bar_init(&lo_full[i], kConvThr / 32);
+      bar_init(&lo_empty[i], 1);
+    }
     bar_init(acc_full, 1);
     bar_init(acc_empty, kEpiThr / 32);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
@@ -294,7 +305,8 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         if (is_tip(op, b)) continue;  // a tip child is a P-column gather in the epilogue: no MMA
         const uint32_t sl = ia % NA, use = ia / NA;
         bar_wait(&a_full[sl], use & 1u);
-        bar_wait(lo_full, ia & 1u);
+        const uint32_t ls = ia % NLO;
+        bar_wait(&lo_full[ls], (ia / NLO) & 1u);
         bar_wait(acc_empty, (ia & 1u) ^ 1u);  // the epilogue drained the previous accumulators
         ++ia;
         fence_after();
@@ -311,7 +323,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         for (int kk = 0; kk < TS / 8; ++kk) {
           const int h = kk >> 2, kin = kk & 3;
           const uint64_t ah = desc_sw128(sbase + SM_A + sl * 32768 + h * 16384 + kin * 32);
-          const uint64_t al = desc_sw128(sbase + SM_ALO + h * 16384 + kin * 32);
+          const uint64_t al = desc_sw128(sbase + SM_ALO + ls * 32768 + h * 16384 + kin * 32);
           const uint64_t bb = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + kin * 32);
           if (h == 0) {
             mma_tf32(tmem, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);
@@ -324,7 +336,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
           }
         }
         commit(&a_empty[sl]);  // child tile, lo tile and matrix tile free once these MMAs completed
-        commit(lo_empty);
+        commit(&lo_empty[ls]);
         commit(&b_empty[bs]);
         commit(acc_full);  // accumulators ready for the epilogue
         TR(4, g);
@@ -340,11 +352,12 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       if (is_tip(op, b) || p0 >= op.p) continue;
       const uint32_t sl = ia % NA, use = ia / NA;
       bar_wait(&a_full[sl], use & 1u);
-      bar_wait(lo_empty, (ia & 1u) ^ 1u);  // the previous internal phase's MMAs read the lo tile
+      const uint32_t ls = ia % NLO;
+      bar_wait(&lo_empty[ls], ((ia / NLO) & 1u) ^ 1u);  // the MMAs NLO internal phases back read this lo tile
       ++ia;
       if (ct == 0) TR(1, g);
       const unsigned char *src = sm + SM_A + sl * 32768;
-      unsigned char *dst = sm + SM_ALO;
+      unsigned char *dst = sm + SM_ALO + ls * 32768;
 #pragma unroll
       for (int u = 0; u < TM * 16 / kConvThr; u += 8) {  // lo of every 16-byte chunk, same swizzled offset
         float4 v[8];
@@ -358,7 +371,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
       __syncwarp();
       if (ct == 0) TR(2, g);
-      if (lane == 0) bar_arrive(lo_full);
+      if (lane == 0) bar_arrive(&lo_full[ls]);
     }
   } else {
     // ================================================================ epilogue
