@@ -500,7 +500,10 @@ def main():
     def measure(cfg, precision, steps, warmup, arms=("level", "sequential")):
         w, scaling = rank_workload(cfg, rank, world)
         n, p, c, s = w.n, w.p, w.c, w.s
-        tl = make(w, "reroot", precision)
+        reuse = cfg == "c4"  # 4,096 x 4 M patterns: liveness buffer reuse (1.1 TB otherwise)
+        if reuse:
+            arms = ()
+        tl = make(w, "reroot", precision, reuse)
         sched = tl.sched
         clocks = ClockSampler(local)
         ms, prof, bm = timed(tl, steps, warmup, clocks)
@@ -579,7 +582,7 @@ def main():
     # per 1,000 reps; reading A6): ops apply the exponents the
     # write pass stored (dest_scale_read) instead of computing new ones
     stored = None
-    if not args.no_secondary and prim["s"] == 4:
+    if not args.no_secondary and prim["s"] == 4 and not reuse:
         tn = TreeLikelihood(w.n, w.p, w.s, w.c, precision=args.precision, device=local,
                             cumulative_scaling=False, cuda_graph=not args.no_graph, stream_ptr=stream.cuda_stream)
         tn.set_model_params(w.model, w.rates, w.cat_weights)
