@@ -11,8 +11,8 @@
 // 8 x 8 x 4 block instead of 256 FMAs and one shared-memory operand load per
 // 32 FMAs instead of per 8.
 //
-// One CTA = one (operation, 128-pattern tile), all categories (the rescale
-// needs max over (c, z)), 16 warps of 32 x 16 (pattern x state) tiles.  DMMA
+// One CTA = one (operation, 64-pattern tile), all categories (the rescale
+// needs max over (c, z)), 8 warps of 32 x 16 (pattern x state) tiles.  DMMA
 // fragment layout (m8n8k4, f64): lane = 4 g + t; A[g][t], B[t][g] (= P[z][x]),
 // D[g][2t + i].  The child tile of an internal child sits in shared memory
 // (68-double rows: a warp's 32 LDS.64 of a fragment are two conflict-free
@@ -32,12 +32,11 @@
 namespace rrl {
 namespace {
 
-constexpr int kS = 61, kSP = 64, kTPD = 128, kThrD = 512;
-constexpr int kRow = 68;  // shared-memory row stride of the A and P tiles (doubles)
+constexpr int kS = 61, kSP = 64, kTPD = 64, kThrD = 256;
+constexpr int kRow = 68;  // shared-memory row stride of the A tile (doubles)
 
 struct DmmaSmem {
   double A[2][kTPD * kRow];  // double-buffered child tiles [pattern][x]
-  double P[2][kSP * kRow];   // the stage's transition matrix [z][x], double-buffered with A
   double mx[4][kTPD];        // per-pattern maxima of the 4 state-quarter warps
   uint8_t st[2][kTPD];       // tip states of both children
 };
@@ -71,16 +70,18 @@ __device__ inline double pow2_neg64(int e) {
 // A tile.  The next internal stage's tile is copied (cp.async) into the other
 // buffer while the current stage's DMMAs run.
 //
-// 16 warps, warp tile 32 patterns x 16 states (wr = warp & 3, wc = warp >> 2):
-// per K-step 4 A fragments and 2 B fragments, all from shared memory (the
-// stage's A tile and P tile are copied together), feed 8 DMMAs.  Measured on
-// configs[3] fp64: 8 x 64 warp tiles with B from L1 were L1-bound (91 %),
-// 32 x 16 tiles with B from L1 reached 72 % L1 and 40 % of the FP64 peak.  A
+// Warp tile 32 patterns x 16 states (wr = warp & 1, wc = warp >> 1): per
+// K-step 4 A fragments (shared memory) and 2 B fragments (the 32 KB P tile,
+// L1-resident) feed 8 DMMAs, so the L1 carries a quarter of the B traffic of
+// an 8 x 64 warp tile (which measured 91 % L1 throughput, the limit).  A
 // thread owns patterns 32 wr + 8 rb + g (rb < 4) and states 16 wc + 8 cb +
 // 2 t + i (cb, i < 2); the per-pattern max over (c, z) is reduced over the 4
 // lanes t by shuffles and over the 4 warps wc through shared memory.
+// (Measured on configs[3] fp64: 8 x 64 warp tiles with B from L1 were L1-bound
+// at 91 %, 7.75 ms per pass; these 32 x 16 tiles 5.17 ms; 16 warps over 128
+// patterns with the P tile staged in shared memory too: 5.68 ms.)
 template <int C>
-__global__ void __launch_bounds__(kThrD, 1)
+__global__ void __launch_bounds__(kThrD, 2)
 k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__restrict__ PT) {
   extern __shared__ __align__(16) unsigned char smem_d[];
   DmmaSmem &sm = *reinterpret_cast<DmmaSmem *>(smem_d);
@@ -93,21 +94,16 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__
   const double *Pg[2] = {static_cast<const double *>(op.P1), static_cast<const double *>(op.P2)};
   const int mat[2] = {op.mat1, op.mat2};
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31, g = lane >> 2, t = lane & 3;
-  const int wr = warp & 3, wc = warp >> 2;
+  const int wr = warp & 1, wc = warp >> 1;
   const int zbase = 16 * wc + 2 * t;  // + 8 cb + i
 
   asm volatile("griddepcontrol.wait;" ::: "memory");
   asm volatile("griddepcontrol.launch_dependents;" :::);
-  auto stage_A = [&](int c, int b, int buf) {  // 128 rows x 512 B + the 64 x 512 B P tile, 16-byte chunks
-    const double *A = static_cast<const double *>(in[b]) + ((size_t)c * p_pad + p0) * kSP;  // rows < p_pad exist
+  auto stage_A = [&](int c, int b, int buf) {  // 64 rows x 512 B, 16-byte chunks; rows beyond p exist (p_pad)
+    const double *A = static_cast<const double *>(in[b]) + ((size_t)c * p_pad + p0) * kSP;
     for (int i = tid; i < kTPD * kSP / 2; i += kThrD) {
       const int r = i / 32, x2 = (i % 32) * 2;
       cp_async16(&sm.A[buf][r * kRow + x2], A + 2 * i);
-    }
-    const double *P = Pg[b] + (size_t)c * kSP * kSP;
-    for (int i = tid; i < kSP * kSP / 2; i += kThrD) {
-      const int z = i / 32, x2 = (i % 32) * 2;
-      cp_async16(&sm.P[buf][z * kRow + x2], P + 2 * i);
     }
     cp_async_commit();
   };
@@ -169,10 +165,10 @@ k_partials_codon_dmma(const DevOp *__restrict__ ops, int p_pad, const double *__
           for (int cb = 0; cb < 2; ++cb) acc[rb][cb][0] = acc[rb][cb][1] = 0.0;
         const double *Ar = &sm.A[buf][(32 * wr + g) * kRow + t];
         // B fragment B[x][z] = P[z][x], z = 16 wc + 8 cb + g, x = 4k + t
-        const double *Pr = &sm.P[buf][(16 * wc + g) * kRow + t];
+        const double *Pr = Pg[b] + (size_t)c * kSP * kSP + (16 * wc + g) * kSP + t;
 #pragma unroll 4
         for (int k = 0; k < kSP / 4; ++k) {
-          const double b0 = Pr[4 * k], b1 = Pr[8 * kRow + 4 * k];
+          const double b0 = __ldg(Pr + 4 * k), b1 = __ldg(Pr + 8 * kSP + 4 * k);
 #pragma unroll
           for (int rb = 0; rb < 4; ++rb) {
             const double a = Ar[(8 * rb) * kRow + 4 * k];

@@ -438,3 +438,38 @@ def test_codon_fp64_dmma_loglik_c3(mode):
     ora = oracle_run(w)
     assert rel(got, ora.lnl) <= LNL_TOL[64], (got, ora.lnl)
     tl.close()
+
+
+def test_stored_factor_read_after_write_in_one_call():
+    """Stored factors are prefetched before a level set's PDL wait only when no
+    op of the call writes a scale buffer that another reads.  Here set-2 ops
+    apply the factor their set-1 child writes in the same call (its buffer
+    zeroed beforehand, so a premature read would apply 0): every output equals
+    pass 1's value rescaled by 2^(e_own - e_child), bit for bit."""
+    from paper_conf_ipps_ayresc18_b200 import rrl as R
+    w = make_workload(tree_kind="random", n=40, p=1_500, model="gtr", c=4, seed=19)
+    tl = gpu_setup(w, "level", 32, cumulative=False)
+    tl.update()
+    n = w.n
+    ops = tl.ops.copy()
+    offs = tl.offsets
+    first = {int(o["dest"]) for o in ops[offs[0]:offs[1]]}
+    before = {int(o["dest"]): (tl.partials(int(o["dest"])), tl.scale(int(o["dest"]) - n)) for o in ops}
+    checked = 0
+    for o in ops[offs[1]:offs[2]]:  # set 2: both children are tips or set-1 nodes
+        ch = int(o["child1"])
+        if ch in first:
+            o["dest_scale_read"] = ch - n
+            o["dest_scale_write"] = -1
+            checked += 1
+    assert checked > 0
+    for v in first:
+        R.rrl_reset_scale_factors(tl.inst, v - n)
+    R.rrl_update_partials(tl.inst, ops, offs)
+    for o in ops[offs[1]:offs[2]]:
+        v, ch = int(o["dest"]), int(o["child1"])
+        if ch in first:
+            L0, e0 = before[v]
+            exp = np.ldexp(L0, (e0 - before[ch][1])[None, :, None])
+            np.testing.assert_array_equal(tl.partials(v), exp)
+    tl.close()
