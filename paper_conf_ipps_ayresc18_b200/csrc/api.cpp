@@ -86,7 +86,6 @@ struct Instance {
   std::vector<int32_t> last_offs;
   std::vector<int32_t> last_ranges;
   std::vector<int> set_tt;               // 61-state fp32: tip-tip ops at the front of each set
-  bool scale_read_safe = true;           // no op of the call reads a scale buffer one writes
   bool ops_valid = false;
   cudaGraphExec_t graph = nullptr;       // replay of the set launches
   cudaStream_t graph_stream = nullptr;
@@ -803,15 +802,6 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
         if (stamp[ops[i].child1] == k || stamp[ops[i].child2] == k)
           return fail(RRL_ERROR_GENERAL, "operation depends on another op of the same set");
     }
-    {  // stored factors (dest_scale_read) may be prefetched before a set's PDL wait
-      std::vector<char> written(I->n_scale > 0 ? I->n_scale : 1, 0);
-      for (int i = 0; i < op_count; ++i)
-        if (ops[i].dest_scale_write >= 0) written[ops[i].dest_scale_write] = 1;
-      I->scale_read_safe = true;
-      for (int i = 0; i < op_count; ++i)
-        if (ops[i].dest_scale_write < 0 && ops[i].dest_scale_read >= 0 && written[ops[i].dest_scale_read])
-          I->scale_read_safe = false;
-    }
     // --- resolve descriptors
     int r = ensure_cap_ops(I, op_count);
     if (r < 0) return r;
@@ -947,7 +937,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
         // tip states may be read before the PDL wait; the matrices too unless this
         // launch directly follows K1 (k = 0: K1 or a host update may be its predecessor)
         e = launch_update_partials_nuc(I->prec, I->c, I->d_ops + offs[k], I->h_ops + offs[k], n, pmax,
-                                       I->p_pad, (k > 0 ? 3 : 1) | (I->scale_read_safe ? 4 : 0), I->stream);
+                                       I->p_pad, k > 0 ? 3 : 1, I->stream);
       } else {
         e = 0;
         int o0 = offs[k], nr = n;  // the ops left for the contraction kernels

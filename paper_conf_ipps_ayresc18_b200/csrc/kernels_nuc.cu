@@ -187,8 +187,7 @@ __device__ inline void matvec(const T *P, const T (&L)[4], T (&v)[4]) {
 
 // Rescale + store of one item (pattern `pat`, category `cat`).  All lanes of
 // the warp must call it (shuffles).  `cum_a`, `cum_b`: children's cumulative
-// exponents (already fetched), 0 when absent; with stored factors
-// (dest_scale_read) `cum_a` carries the prefetched factor to apply.
+// exponents (already fetched), 0 when absent.
 template <typename T, int C>
 __device__ inline void finish_item(const DevOp &op, T (&r)[4], bool valid, unsigned pat, int cat,
                                    int cum_a, int cum_b, T *out_item) {
@@ -200,7 +199,8 @@ __device__ inline void finish_item(const DevOp &op, T (&r)[4], bool valid, unsig
     if (e != 0) scale_pow2(r, e);
     if (valid && cat == 0) op.scale_out[pat] = e + cum_a + cum_b;
   } else if (op.scale_in != nullptr) {
-    if (cum_a != 0) scale_pow2(r, cum_a);
+    const int e = valid ? __ldg(op.scale_in + pat) : 0;
+    if (e != 0) scale_pow2(r, e);
   }
   if (valid) V4<T>::st(out_item, r);
 }
@@ -235,9 +235,8 @@ __device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
 // `early` (host-decided): bit 0 -- tip states may be read before griddepcontrol.wait
 // (only host copies write them); bit 1 -- so may the transition matrices (K1 is
 // not this launch's immediate predecessor, so it completed before the previous
-// level set passed its own wait); bit 2 -- so may stored scale factors (no op
-// of the call writes a scale buffer that one reads).  Only the previous level
-// set's partials and exponents must wait.
+// level set passed its own wait).  Only the previous level set's partials and
+// exponents must wait.
 template <typename T, int C, int U>
 __global__ void __launch_bounds__(kLatThreads, sizeof(T) == 4 ? kLatencyMinBlocks : kLatencyMinBlocks64)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int early) {
@@ -270,20 +269,13 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
       }
     }
   };
-  // first chunk's tip states (and rows) in flight while the previous level set
-  // finishes; stored scale factors too (dest_scale_read) when the host found no
-  // op of this call writing a scale buffer another op reads (early bit 2: they
-  // come from an earlier pass, complete before the previous set's own wait)
-  const bool read_sc = op.scale_out == nullptr && op.scale_in != nullptr;
-  const bool pre_sc = read_sc && (early & 4);
+  // first chunk's tip states (and rows) in flight while the previous level set finishes
   unsigned s1p[U], s2p[U];
-  int sinp[U];
+  if (early & 1) {
 #pragma unroll
-  for (int j = 0; j < U; ++j) {
-    const unsigned item = (unsigned)blockIdx.x * (kLatThreads * U) + threadIdx.x + j * kLatThreads;
-    const bool valid = item < nitems && (int)blockIdx.x < nchunks;
-    sinp[j] = (pre_sc && valid) ? __ldg(op.scale_in + item / C) : 0;
-    if (early & 1) {
+    for (int j = 0; j < U; ++j) {
+      const unsigned item = (unsigned)blockIdx.x * (kLatThreads * U) + threadIdx.x + j * kLatThreads;
+      const bool valid = item < nitems && (int)blockIdx.x < nchunks;
       s1p[j] = (tip1 && valid) ? (unsigned)__ldg(S1g + item / C) : 4u;
       s2p[j] = (tip2 && valid) ? (unsigned)__ldg(S2g + item / C) : 4u;
     }
@@ -335,8 +327,6 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
       }
       ca[j] = (scale_w && valid && cat == 0 && op.cum1 != nullptr) ? __ldg(op.cum1 + pat) : 0;
       cb[j] = (scale_w && valid && cat == 0 && op.cum2 != nullptr) ? __ldg(op.cum2 + pat) : 0;
-      if (read_sc)  // the stored factor to apply rides in ca
-        ca[j] = (pre_sc && chunk == (int)blockIdx.x) ? sinp[j] : (valid ? __ldg(op.scale_in + pat) : 0);
     }
     if constexpr (!kRegP) {
       if (!tables) {  // block-uniform, first chunk only
