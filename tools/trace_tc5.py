@@ -25,7 +25,8 @@ LIB = os.path.join(ROOT, "paper_conf_ipps_ayresc18_b200", "_lib", "librrl-trace.
 
 
 def main():
-    env = dict(os.environ, RRL_BUILD_TAG="trace", RRL_NVCC_EXTRA="-DRRL_TC5_TRACE")
+    extra = os.environ.get("TRACE_EXTRA", "")  # e.g. "-DRRL_TC5_NLO=2" (ring-depth variants)
+    env = dict(os.environ, RRL_BUILD_TAG="trace", RRL_NVCC_EXTRA=("-DRRL_TC5_TRACE " + extra).strip())
     subprocess.run([sys.executable, "-m", "paper_conf_ipps_ayresc18_b200.build"], env=env, check=True,
                    cwd=ROOT)
     os.environ["RRL_LIB_PATH"] = LIB
