@@ -75,17 +75,41 @@ constexpr int kThr = 15 * 32;
 #ifndef RRL_TC5_NB
 #define RRL_TC5_NB 2
 #endif
+// Build knobs, all measured on configs[3] fp32 (updatePartials per pass):
+//  * RRL_TC5_DIRECT_STORE=1: write-back by direct 16-byte stores from the
+//    epilogue (a thread's row is 128 contiguous bytes, a warp instruction
+//    touches 32 rows) instead of the swizzled staging tile drained by TMA
+//    stores, freeing 32 KB for a fourth child tile in flight: 2.03 ms vs
+//    1.535 -- the uncoalesced stores cost far more than the deeper ring wins;
+//  * RRL_TC5_NLO=2 (a second lo tile, so the converters run under the
+//    previous phase's MMAs), RRL_TC5_NB=3 (a third matrix slot), RRL_TC5_ACC4=1
+//    (round 1's [main_h | corr_h] accumulators: per K-step one N = 128 + one
+//    N = 64 MMA instead of K-half 1's three N = 64): 1.536-1.543 ms, no change.
+// The phase timeline (tools/trace_tc5.py) puts the MMAs of an internal phase
+// at ~1,350 cycles (24 tf32 MMAs) and a child tile's TMA load from HBM at
+// ~2.5 K cycles; the period stays ~2.4 K cycles per phase whichever ring
+// is deepened.
+#ifndef RRL_TC5_DIRECT_STORE
+#define RRL_TC5_DIRECT_STORE 0
+#endif
 constexpr int NLO = RRL_TC5_NLO;  // lo tiles (2: the converters run under the previous phase's MMAs)
 constexpr int NB = RRL_TC5_NB;    // matrix tiles (3: a tip phase's P tile lands while the previous one is read)
-constexpr int NA = 6 - NLO - NB;  // child tiles; 6 x 32 KB of rings + the staging tile fit 227 KB
+constexpr int NA = (RRL_TC5_DIRECT_STORE ? 7 : 6) - NLO - NB;  // child tiles: 7 x 32 KB of rings fit 227 KB
 constexpr int SM_A = 0, SM_ALO = NA * 32768, SM_B = SM_ALO + NLO * 32768, SM_S1 = SM_B + NB * 32768;
 static_assert(NA >= 1 && 2 * (NA + NB + NLO) + 2 <= 16, "ring sizes / mbarrier slots");
-constexpr int SMEM_MX = SM_S1 + TM * TS * 4;           // row maxima / scale [2][128]
+constexpr int SMEM_MX = SM_S1 + (RRL_TC5_DIRECT_STORE ? 0 : TM * TS * 4);  // row maxima / scale [2][128]
 constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 16 mbarriers
 constexpr int SMEM_TMEM = SMEM_BAR + 16 * 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 16;
-constexpr int kTmemCols = 512;    // [main_0 | corr | main_1] (3 x 64) ...
-constexpr int kProdCol = 3 * TS;  // ... + one 64-column slot per category (the unscaled product)
+#ifndef RRL_TC5_ACC4
+#define RRL_TC5_ACC4 0
+#endif
+constexpr int kTmemCols = 512;
+// accumulators: ACC4 [main_0 | corr_0 | main_1 | corr_1] (4 x 64: per K-half one
+// N = 128 MMA A_hi.[P_hi|P_lo] + one N = 64 A_lo.P_hi), else [main_0 | corr |
+// main_1] (3 x 64: K-half 1 as three N = 64 MMAs); then one 64-column slot per
+// category (the unscaled product)
+constexpr int kProdCol = (RRL_TC5_ACC4 ? 4 : 3) * TS;
 
 __device__ inline uint32_t sa(const void *p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
 __device__ inline uint64_t desc_sw128(uint32_t saddr) {  // K-major, 128-byte swizzle, 8-row atoms of 1 KB
@@ -325,7 +349,11 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
           const uint64_t ah = desc_sw128(sbase + SM_A + sl * 32768 + h * 16384 + kin * 32);
           const uint64_t al = desc_sw128(sbase + SM_ALO + ls * 32768 + h * 16384 + kin * 32);
           const uint64_t bb = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + kin * 32);
-          if (h == 0) {
+          if (RRL_TC5_ACC4) {
+            const uint32_t d = tmem + (uint32_t)(h * 2 * TS);
+            mma_tf32(d, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);  // [main_h | corr_h]
+            mma_tf32(d + TS, al, bb, idesc_tf32(TS), 1u);                // corr_h += A_lo P_hi
+          } else if (h == 0) {
             mma_tf32(tmem, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);
             mma_tf32(tmem + TS, al, bb, idesc_tf32(TS), 1u);
           } else {
@@ -408,12 +436,24 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     // swizzled layout, and hand it to an asynchronous TMA bulk tensor store
     float sc_prev = 0.f;
     int prev_y = 0, prev_buf = 0;
+    float *prev_dst = nullptr;  // direct write-back: row p0 of category 0 of the previous tile's output
     bool have_prev = false;
     auto drain = [&](int cat) {
       float w0[16], w1[16];
       tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), w0);
       tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), w1);
       tmem_wait_ld();
+      if (RRL_TC5_DIRECT_STORE) {
+        float4 *dst = reinterpret_cast<float4 *>(prev_dst + ((size_t)cat * p_pad + r) * TS + h * 32);
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          dst[k] = make_float4(w0[4 * k] * sc_prev, w0[4 * k + 1] * sc_prev, w0[4 * k + 2] * sc_prev,
+                               w0[4 * k + 3] * sc_prev);
+          dst[4 + k] = make_float4(w1[4 * k] * sc_prev, w1[4 * k + 1] * sc_prev, w1[4 * k + 2] * sc_prev,
+                                   w1[4 * k + 3] * sc_prev);
+        }
+        return;
+      }
       if (tid == 0) bulk_wait_read0();  // the previous store has read the staging tile
       named_sync(1, kEpiThr);
 #pragma unroll
@@ -497,13 +537,21 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         if (tid == 0) TR(7, g);
 #pragma unroll
         for (int q = 0; q < 2; ++q) {
-          float m0[16], cc[16], m1[16];
+          float m0[16], cc[16], m1[16];  // main_0 (columns 0-63), a correction (64-127), main_1 (128-191)
           tmem_ld16(tl + 0 * TS + q * 16, m0);
           tmem_ld16(tl + 1 * TS + q * 16, cc);
           tmem_ld16(tl + 2 * TS + q * 16, m1);
-          tmem_wait_ld();
+          if (RRL_TC5_ACC4) {  // + corr_1 (192-255)
+            float c1[16];
+            tmem_ld16(tl + 3 * TS + q * 16, c1);
+            tmem_wait_ld();
 #pragma unroll
-          for (int i = 0; i < 16; ++i) dv[q * 16 + i] = (m0[i] + m1[i]) + cc[i];
+            for (int i = 0; i < 16; ++i) dv[q * 16 + i] = (m0[i] + m1[i]) + (cc[i] + c1[i]);
+          } else {
+            tmem_wait_ld();
+#pragma unroll
+            for (int i = 0; i < 16; ++i) dv[q * 16 + i] = (m0[i] + m1[i]) + cc[i];
+          }
         }
         fence_before();
         __syncwarp();
@@ -550,6 +598,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       sc_prev = valid ? mx[r] : 0.f;  // padding rows of the tile are written as zeros
       prev_y = op.pat0 + p0;
       prev_buf = op.bufd;
+      prev_dst = static_cast<float *>(op.out) + (size_t)p0 * TS;
       have_prev = true;
       if (tid == 0) TR(6, g);
       m = 0.f;
