@@ -25,13 +25,7 @@ import numpy as np
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 
-VARIANTS = [("simt", {}), ("tc5", {})]
-
-
-def set_env(env):
-    for k in ("RRL_CODON_KERNEL", "RRL_TCC_NMAIN"):
-        os.environ.pop(k, None)
-    os.environ.update(env)
+VARIANTS = ("simt", "tc5")
 
 
 def one_op(R, simt, rng):
@@ -109,15 +103,13 @@ def main():
     from paper_conf_ipps_ayresc18_b200 import rrl as R
     out = {}
     ctx = None
-    for name, env in VARIANTS:
-        set_env(env)
+    for name in VARIANTS:
         simt = name == "simt"
         op = one_op(R, simt, np.random.default_rng(0))
         by_h, w, rt, ora = depth_errors(simt)
         ctx = (w, rt, ora)
         out[name] = {"one_op": op, "c3_node_error_by_height": by_h, "c3_max": max(by_h.values())}
         print(name, json.dumps(op), f"c3 max {max(by_h.values()):.3e} at h27 {by_h.get(27, 0):.3e}", flush=True)
-    set_env({})
     fl = fp32_floor(*ctx)
     out["fp32_emulation_floor"] = {"c3_node_error_by_height": fl, "c3_max": max(fl.values())}
     print("fp32 floor", f"c3 max {max(fl.values()):.3e}", flush=True)
