@@ -105,10 +105,12 @@ class TreeLikelihood:
         return R.rrl_schedule_cost(self.n, sch["ops"], sch["set_offsets"], self.p, self.s, self.c,
                                    self.precision, self.launch_us, self.hbm_gbs, self.l2_bytes)
 
-    def set_tree(self, parent, blen, mode: str = "reroot", reuse_buffers: bool = False):
-        """mode: "sequential" | "level" | "reroot" | "auto" -- auto reroots only
-        when the cost model predicts the rerooted schedule to be faster
-        (NEXT-4; PAPER.md:270, :288)."""
+    def set_tree(self, parent, blen, mode: str = "auto", reuse_buffers: bool = False):
+        """mode: "sequential" | "level" | "reroot" | "auto" (default) -- auto
+        reroots only when the cost model predicts the rerooted schedule to be
+        faster (NEXT-4): every measured point of the
+        1,024-pectinate sweep below 10^6 fp32 patterns, not that one
+        (profiles/r02_reroot_sweep.json)."""
         if reuse_buffers and not self.cumulative:
             # recycled buffers recycle their scale buffers too: per-node exponents
             # of consumed children would be overwritten before K5 sums them

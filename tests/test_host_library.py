@@ -233,3 +233,66 @@ def test_update_schedule_no_change_and_errors(R):
         R.rrl_tree_spr(30, t.parent, t.blen, a, 0 if a != 0 else 1)   # parent of prune node is the root
     with pytest.raises(R.RRLError):
         R.rrl_tree_nni(30, t.parent, t.blen, 3, 0)                     # a tip is no internal edge
+
+
+# ------------------------------------------------------------------ NEXT-4 cost model (host only)
+def test_schedule_cost_closed_forms(R):
+    """rrl_schedule_cost against closed forms of a pectinate tree (PAPER.md:270,
+    :288; DESIGN.md §9 "NEXT-4"): with no L2 credit the pass costs every set's
+    launch plus every byte once -- n-1 outputs, n-2 internal children, n tip
+    children; with infinite bandwidth it is the set count times the launch."""
+    n, p, c, s = 64, 1000, 4, 4
+    t = make_tree("pectinate", n, seed=3)
+    for prec in (32, 64):
+        v = c * s * prec // 8
+        for mode, sets in (("level", n - 1), ("reroot", n // 2)):
+            sch = R.rrl_reroot_and_schedule(n, t.parent, t.blen, mode)
+            assert sch["set_count"] == sets
+            bytes_ = p * ((n - 1) * (v + 4) + (n - 2) * (v + 4) + n * 1)
+            got = R.rrl_schedule_cost(n, sch["ops"], sch["set_offsets"], p, s, c, prec, 2.0, 1000.0, 0.0)
+            assert got == pytest.approx(sets * 2.0 + bytes_ / 1e12 * 1e6, rel=1e-12)
+            got = R.rrl_schedule_cost(n, sch["ops"], sch["set_offsets"], p, s, c, prec, 3.0, 1e300, 0.0)
+            assert got == pytest.approx(sets * 3.0, rel=1e-12)
+
+
+def test_schedule_cost_l2_credit(R):
+    """A chain (one op per set) whose outputs fit in L2 reads every internal
+    child from L2: the credit removes exactly those reads; outputs bigger than
+    L2 get none."""
+    n, p, c, s = 32, 1000, 4, 4
+    t = make_tree("pectinate", n, seed=1)
+    sch = R.rrl_reroot_and_schedule(n, t.parent, t.blen, "level")
+    v = c * s * 4 + 4
+    full = R.rrl_schedule_cost(n, sch["ops"], sch["set_offsets"], p, s, c, 32, 0.0, 1000.0, 0.0)
+    huge = R.rrl_schedule_cost(n, sch["ops"], sch["set_offsets"], p, s, c, 32, 0.0, 1000.0, 1e30)
+    tiny = R.rrl_schedule_cost(n, sch["ops"], sch["set_offsets"], p, s, c, 32, 0.0, 1000.0, v * p / 2)
+    assert huge == pytest.approx(full - (n - 2) * v * p / 1e6, rel=1e-9)
+    assert tiny == pytest.approx(full, rel=1e-12)
+
+
+def test_schedule_cost_predicts_measured_crossover(R):
+    """The B200 parameters the engine's auto mode uses (engine.py) pick the
+    rerooted 1,024-pectinate schedule where it measured faster and the original
+    chain at 10^6 fp32 patterns, where it measured 0.88x
+    (profiles/r02_reroot_sweep.json)."""
+    n = 1024
+    t = make_tree("pectinate", n, seed=1)
+    lv = R.rrl_reroot_and_schedule(n, t.parent, t.blen, "level", True)
+    rr = R.rrl_reroot_and_schedule(n, t.parent, t.blen, "reroot", True)
+
+    def cost(sch, p):
+        return R.rrl_schedule_cost(n, sch["ops"], sch["set_offsets"], p, 4, 4, 32, 2.0, 6225.0, 126e6)
+    for p in (512, 4096, 10_000, 100_000):
+        assert cost(rr, p) < cost(lv, p), p
+    assert cost(lv, 1_000_000) < cost(rr, 1_000_000)
+
+
+def test_schedule_cost_rejects_bad_input(R):
+    t = make_tree("random", 10, seed=1)
+    sch = R.rrl_reroot_and_schedule(10, t.parent, t.blen, "level")
+    bad = sch["set_offsets"].copy()
+    bad[-1] -= 1
+    with pytest.raises(RuntimeError):
+        R.rrl_schedule_cost(10, sch["ops"], bad, 100, 4, 4, 32)
+    with pytest.raises(RuntimeError):
+        R.rrl_schedule_cost(10, sch["ops"], sch["set_offsets"], 100, 4, 4, 16)
