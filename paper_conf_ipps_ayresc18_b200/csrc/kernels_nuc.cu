@@ -66,6 +66,15 @@ constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 #ifndef RRL_LAT_PDL_EARLY
 #define RRL_LAT_PDL_EARLY 1
 #endif
+#ifndef RRL_LAT_U  // items per thread on the latency path
+#define RRL_LAT_U 1
+#endif
+#ifndef RRL_LAT_PDL_TOP
+#define RRL_LAT_PDL_TOP 0
+#endif
+#ifndef RRL_LAT_TLB_PREFETCH
+#define RRL_LAT_TLB_PREFETCH 0
+#endif
 #ifndef RRL_LAT_THREADS
 #define RRL_LAT_THREADS 128
 #endif
@@ -153,19 +162,27 @@ __device__ inline void scale_pow2(double (&r)[4], int e) {
 }
 
 // Shared-memory transition tables of one operation: [branch][cat][kPTab].
-template <typename T, int C>
+template <typename T, int C, int NT>  // NT = blockDim.x (compile-time: no runtime trip-count division)
 __device__ inline void load_ptables(T (*sP)[C][kPTab], const DevOp &op) {
-  for (int t = threadIdx.x; t < 2 * C * 16; t += blockDim.x) {
-    const int b = t / (C * 16), r = t % (C * 16), c = r / 16, zx = r % 16;
-    const T v = static_cast<const T *>(b == 0 ? op.P1 : op.P2)[r];
-    sP[b][c][zx] = v;                                // row-major P[z][x]
-    sP[b][c][16 + (zx % 4) * 4 + zx / 4] = v;        // column x at 16 + 4x
+#pragma unroll
+  for (int t0 = 0; t0 < 2 * C * 16; t0 += NT) {
+    const int t = t0 + threadIdx.x;
+    if (t < 2 * C * 16) {
+      const int b = t / (C * 16), r = t % (C * 16), c = r / 16, zx = r % 16;
+      const T v = __ldg(static_cast<const T *>(b == 0 ? op.P1 : op.P2) + r);
+      sP[b][c][zx] = v;                                // row-major P[z][x]
+      sP[b][c][16 + (zx % 4) * 4 + zx / 4] = v;        // column x at 16 + 4x
+    }
   }
   __syncthreads();
-  for (int t = threadIdx.x; t < 2 * C * 4; t += blockDim.x) {
-    const int b = t / (C * 4), r = t % (C * 4), c = r / 4, z = r % 4;
-    const T *row = &sP[b][c][z * 4];
-    sP[b][c][32 + z] = row[0] + row[1] + row[2] + row[3];  // "column 4" = row sums
+#pragma unroll
+  for (int t0 = 0; t0 < 2 * C * 4; t0 += NT) {
+    const int t = t0 + threadIdx.x;
+    if (t < 2 * C * 4) {
+      const int b = t / (C * 4), r = t % (C * 4), c = r / 4, z = r % 4;
+      const T *row = &sP[b][c][z * 4];
+      sP[b][c][32 + z] = row[0] + row[1] + row[2] + row[3];  // "column 4" = row sums
+    }
   }
   __syncthreads();
 }
@@ -206,6 +223,24 @@ __device__ inline void finish_item(const DevOp &op, T (&r)[4], bool valid, unsig
 }
 
 __device__ inline void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ inline void prefetch_l2(const void *p) { asm volatile("prefetch.global.L2 [%0];" ::"l"(p)); }
+#ifdef RRL_LAT_TRACE  // dev build only (tools/trace_latency.py): per-CTA globaltimer stamps
+// per-SM slots (no single contended counter): record k of SM s at [s * kLatSlots + k]
+constexpr unsigned kLatSlots = 1024;
+__device__ unsigned long long g_lat_trace[160 * kLatSlots][4];
+__device__ unsigned int g_lat_n[160];
+__device__ inline unsigned long long gtime() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t)::"memory");
+  return t;
+}
+// stamp issued after x is available (in-order issue: the add waits for x)
+__device__ inline unsigned long long gtime_after(float x) {
+  unsigned long long t;
+  asm volatile("{.reg .f32 d; add.f32 d, %1, 0f00000000; mov.u64 %0, %%globaltimer;}" : "=l"(t) : "f"(x) : "memory");
+  return t;
+}
+#endif
 __device__ inline void pdl_launch() { asm volatile("griddepcontrol.launch_dependents;" :::); }
 
 // ============================================================ latency path
@@ -237,10 +272,22 @@ __device__ inline void matvec_r(const T (&P)[16], const T (&L)[4], T (&v)[4]) {
 // not this launch's immediate predecessor, so it completed before the previous
 // level set passed its own wait).  Only the previous level set's partials and
 // exponents must wait.
-template <typename T, int C, int U>
+template <typename T, int C, int U, bool INL>
 __global__ void __launch_bounds__(kLatThreads, sizeof(T) == 4 ? kLatencyMinBlocks : kLatencyMinBlocks64)
 k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int early) {
-  const DevOp &op = (pack.n <= kInline) ? pack.inl[blockIdx.y] : pack.ops[blockIdx.y];
+#if RRL_LAT_PDL_TOP
+  pdl_launch();
+#endif
+  // The descriptor by value: inline descriptors are read from the parameter
+  // bank (LDC, register-indexed); a reference selecting between the bank and
+  // global memory would turn every field into a generic load, and the ones
+  // first used after griddepcontrol.wait (cumulative-exponent pointers) into
+  // an extra dependent round trip.
+  // INL is a separate kernel: with a runtime branch the compiler loads both
+  // sources and selects, i.e. every warp also reads the global copy.
+  DevOp op;
+  if constexpr (INL) op = pack.inl[blockIdx.y];
+  else op = pack.ops[blockIdx.y];
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
   const int cat = threadIdx.x % C;  // kLatThreads is a multiple of C
   const T *__restrict__ P1g = static_cast<const T *>(op.P1) + cat * 16;
@@ -253,6 +300,10 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
   const bool scale_w = op.scale_out != nullptr;
   const unsigned nitems = (unsigned)op.p * C;  // this operation's pattern range
   (void)p;
+#ifdef RRL_LAT_TRACE
+  const unsigned long long t_entry = gtime();
+  unsigned long long t_ld = 0;
+#endif
 
   // fp32: each thread holds its category's rows in registers.  fp64: the rows
   // would cost 64 registers, so the block stages the tables in shared memory
@@ -284,17 +335,41 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
   bool tables = kRegP;
   if constexpr (!kRegP) {
     if (early & 2) {  // K1 completed before the previous set: the tables can be staged before the wait
-      load_ptables<T, C>(sP, op);
+      load_ptables<T, C, kLatThreads>(sP, op);
       tables = true;
     }
   }
 
-#if RRL_LAT_PDL_EARLY
+#if RRL_LAT_TLB_PREFETCH
+  // Address-translation warm-up before the wait: one L2 prefetch per warp into
+  // each page this warp will touch.  No value is read (a prefetch only moves
+  // a line into L2, the coherence point, so a later write by the previous set
+  // still lands there); the children are consumed after griddepcontrol.wait.
+  if ((threadIdx.x & 31) == 0 && (int)blockIdx.x < nchunks) {
+    const unsigned item = (unsigned)blockIdx.x * (kLatThreads * U) + threadIdx.x;
+    if (item < nitems) {
+      if (!tip1) prefetch_l2(L1g + (size_t)item * 4);
+      if (!tip2) prefetch_l2(L2g + (size_t)item * 4);
+      prefetch_l2(out + (size_t)item * 4);
+      if (scale_w) {
+        prefetch_l2(op.scale_out + item / C);
+        if (op.cum1 != nullptr) prefetch_l2(op.cum1 + item / C);
+        if (op.cum2 != nullptr) prefetch_l2(op.cum2 + item / C);
+      }
+    }
+  }
+#endif
+#if RRL_LAT_PDL_TOP
+  pdl_wait();  // everything above overlaps the previous level set
+#elif RRL_LAT_PDL_EARLY
   pdl_launch();
   pdl_wait();  // everything above overlaps the previous level set
 #else
   pdl_wait();  // everything above overlaps the previous level set
   pdl_launch();
+#endif
+#ifdef RRL_LAT_TRACE
+  const unsigned long long t_wait = gtime();
 #endif
 
   if (!(early & 2)) load_rows();
@@ -330,7 +405,7 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
     }
     if constexpr (!kRegP) {
       if (!tables) {  // block-uniform, first chunk only
-        load_ptables<T, C>(sP, op);
+        load_ptables<T, C, kLatThreads>(sP, op);
         tables = true;
       }
     }
@@ -350,9 +425,30 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
       }
 #pragma unroll
       for (int z = 0; z < 4; ++z) r[z] = v1[z] * v2[z];
+#ifdef RRL_LAT_TRACE
+      if (j == 0 && threadIdx.x == 0 && t_ld == 0) t_ld = gtime_after((float)r[0] + (float)ca[0] + (float)cb[0]);
+#endif
       finish_item<T, C>(op, r, valid, pat, cat, ca[j], cb[j], out + (size_t)item * 4);
     }
   }
+#ifdef RRL_LAT_TRACE
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    unsigned smid;
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    const unsigned long long t_end = gtime();
+    const unsigned k = smid < 160 ? atomicAdd(&g_lat_n[smid], 1u) : kLatSlots;
+    if (k < kLatSlots) {
+      const unsigned long long q = smid * kLatSlots + k;
+      const DevOp &op0 = INL ? pack.inl[0] : pack.ops[0];  // identifies the level set
+      g_lat_trace[q][0] = (unsigned long long)op0.out;
+      g_lat_trace[q][1] = (unsigned long long)blockIdx.x | ((unsigned long long)blockIdx.y << 16) |
+                          ((unsigned long long)smid << 32);
+      g_lat_trace[q][2] = t_entry;
+      g_lat_trace[q][3] = (t_wait - t_entry) | ((t_ld ? t_ld - t_entry : 0ull) << 21) | ((t_end - t_entry) << 42);
+    }
+  }
+#endif
 }
 
 // ============================================================ fused pass
@@ -609,7 +705,7 @@ template <typename T, int C>
 __device__ inline void load_ptables_consumers(T (*sP)[C][kPTab], const DevOp &op) {
   for (int t = threadIdx.x; t < 2 * C * 16; t += kThreads) {
     const int b = t / (C * 16), r = t % (C * 16), c = r / 16, zx = r % 16;
-    const T v = static_cast<const T *>(b == 0 ? op.P1 : op.P2)[r];
+    const T v = __ldg(static_cast<const T *>(b == 0 ? op.P1 : op.P2) + r);
     sP[b][c][zx] = v;
     sP[b][c][16 + (zx % 4) * 4 + zx / 4] = v;
   }
@@ -879,7 +975,8 @@ int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, in
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
-    cudaError_t e = cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U>, pack, p, nchunks, early);
+    cudaError_t e = pack.n <= kInline ? cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U, true>, pack, p, nchunks, early)
+                                      : cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U, false>, pack, p, nchunks, early);
     if (e != cudaSuccess) return (int)e;
   }
   return 0;
@@ -896,12 +993,12 @@ int launch_latency(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, int 
   int &resident = resident_dev[device_slot()];
   if (resident <= 0) {
     int per_sm = 1, dev = 0, nsm = 148;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, 1>, kLatThreads, 0);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k_partials_nuc<T, C, RRL_LAT_U, true>, kLatThreads, 0);
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
     resident = (per_sm > 0 ? per_sm : 1) * nsm;
   }
-  return launch_latency_u<T, C, 1>(d_ops, h_ops, nops, p, resident, early, st);
+  return launch_latency_u<T, C, RRL_LAT_U>(d_ops, h_ops, nops, p, resident, early, st);
 }
 
 template <typename T, int C>
@@ -1036,3 +1133,16 @@ int launch_update_partials_nuc(int prec, int c, const DevOp *d_ops, const DevOp 
 }
 
 }  // namespace rrl
+
+#ifdef RRL_LAT_TRACE
+// Dev build only: copy out and reset the latency-path trace.  rec: [160 * 1024][4]
+// (SM s's records at s * 1024, count cnt[s]); returns 0 or -1.
+extern "C" int rrl_debug_lat_trace(unsigned long long *rec, unsigned *cnt /*[160]*/) {
+  if (cudaDeviceSynchronize() != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(cnt, rrl::g_lat_n, sizeof(rrl::g_lat_n)) != cudaSuccess) return -1;
+  if (cudaMemcpyFromSymbol(rec, rrl::g_lat_trace, sizeof(rrl::g_lat_trace)) != cudaSuccess) return -1;
+  static const unsigned z[160] = {};
+  if (cudaMemcpyToSymbol(rrl::g_lat_n, z, sizeof(z)) != cudaSuccess) return -1;
+  return 0;
+}
+#endif
