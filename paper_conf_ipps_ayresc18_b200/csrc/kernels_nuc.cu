@@ -40,21 +40,32 @@ namespace rrl {
 namespace {
 
 constexpr int kThreads = 256;
-constexpr int kInline = 8;
+#ifndef RRL_LAT_INLINE
+#define RRL_LAT_INLINE 8
+#endif
+constexpr int kInline = RRL_LAT_INLINE;
 // Latency path: the transition tables live in shared memory (staged before
 // griddepcontrol.wait when K1 is not the immediate predecessor) instead of 32
-// registers per thread, and the CTA is held to 5 resident per SM (48
+// registers per thread, and the CTA is held to 12 resident per SM (42
 // registers, no spills), so the next level set's CTAs (2.1 per SM at
 // configs[1]) are resident beside the current set's under programmatic
 // dependent launch and finish their whole prologue before its wait.
-// Measured on configs[1] (updatePartials per pass, fp32): rows in registers,
-// 80 registers 0.173 ms; tables in shared memory, 256-thread CTAs at 3 / 4 /
-// 5 / 6 per SM 0.163 / 0.178 (spills) / 0.145 / 0.169 ms; 128-thread CTAs at
-// 10 per SM (48 registers) 0.143 ms; 512-thread CTAs 0.176-0.183 ms.  fp64
-// (tables in shared memory already) keeps 3 CTAs per SM: at 5 it spills and is
-// no faster (0.214 ms).
+// Measured on configs[1] (updatePartials per pass, fp32; round 1): rows in
+// registers, 80 registers 0.173 ms; tables in shared memory, 256-thread CTAs
+// at 3 / 4 / 5 / 6 per SM 0.163 / 0.178 (spills) / 0.145 / 0.169 ms;
+// 128-thread CTAs at 10 per SM 0.143 ms; 512-thread CTAs 0.176-0.183 ms.
+// Round 2 (after the descriptor and table-staging fixes, 0.117-0.119 ms):
+// 8 / 10 / 12 / 14 / 16 CTAs per SM 0.145 / 0.119 / 0.117 / 0.119 / 0.119 ms;
+// 2 items per thread 0.153; 64- or 256-thread CTAs 0.162 / 0.132;
+// launch_dependents at the top of the kernel 0.145; an L2 prefetch of the
+// children's pages before the wait 0.163; tip states read after the wait
+// 0.151; the tip-state array bulk-prefetched into L2 by the first set 0.157
+// (one SM's bulk engine streams 1.3 MB while that CTA cannot retire); 2 or 4
+// inline descriptors instead of 8 0.117 / 0.118 (the pointer path for a
+// 2-operation set: 0.147).  fp64 (tables in shared memory already) keeps 3
+// CTAs per SM: at 5 it spills and is no faster.
 #ifndef RRL_LAT_MINB
-#define RRL_LAT_MINB 10
+#define RRL_LAT_MINB 12
 #endif
 #ifndef RRL_LAT_PSMEM
 #define RRL_LAT_PSMEM 1
@@ -68,6 +79,12 @@ constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 #endif
 #ifndef RRL_LAT_U  // items per thread on the latency path
 #define RRL_LAT_U 1
+#endif
+#ifndef RRL_LAT_ABL  // timing ablations (dev builds only; results are wrong): 1 no child exponents, 2 no rescale
+#define RRL_LAT_ABL 0
+#endif
+#ifndef RRL_LAT_PIN
+#define RRL_LAT_PIN 0
 #endif
 #ifndef RRL_LAT_PDL_TOP
 #define RRL_LAT_PDL_TOP 0
@@ -164,24 +181,20 @@ __device__ inline void scale_pow2(double (&r)[4], int e) {
 // Shared-memory transition tables of one operation: [branch][cat][kPTab].
 template <typename T, int C, int NT>  // NT = blockDim.x (compile-time: no runtime trip-count division)
 __device__ inline void load_ptables(T (*sP)[C][kPTab], const DevOp &op) {
-#pragma unroll
-  for (int t0 = 0; t0 < 2 * C * 16; t0 += NT) {
-    const int t = t0 + threadIdx.x;
-    if (t < 2 * C * 16) {
-      const int b = t / (C * 16), r = t % (C * 16), c = r / 16, zx = r % 16;
-      const T v = __ldg(static_cast<const T *>(b == 0 ? op.P1 : op.P2) + r);
-      sP[b][c][zx] = v;                                // row-major P[z][x]
-      sP[b][c][16 + (zx % 4) * 4 + zx / 4] = v;        // column x at 16 + 4x
-    }
-  }
-  __syncthreads();
+  // one thread per row P[c][z][.] of either branch: one vector load, the row,
+  // its 4 column entries and its sum written straight away, one barrier
 #pragma unroll
   for (int t0 = 0; t0 < 2 * C * 4; t0 += NT) {
     const int t = t0 + threadIdx.x;
     if (t < 2 * C * 4) {
       const int b = t / (C * 4), r = t % (C * 4), c = r / 4, z = r % 4;
-      const T *row = &sP[b][c][z * 4];
-      sP[b][c][32 + z] = row[0] + row[1] + row[2] + row[3];  // "column 4" = row sums
+      T row[4];
+      V4<T>::ld(static_cast<const T *>(b == 0 ? op.P1 : op.P2) + r * 4, row);
+      T *tab = &sP[b][c][0];
+      V4<T>::st(tab + z * 4, row);                        // row-major P[z][x]
+#pragma unroll
+      for (int x = 0; x < 4; ++x) tab[16 + x * 4 + z] = row[x];  // column x at 16 + 4x
+      tab[32 + z] = row[0] + row[1] + row[2] + row[3];    // "column 4" = row sums
     }
   }
   __syncthreads();
@@ -288,6 +301,16 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
   DevOp op;
   if constexpr (INL) op = pack.inl[blockIdx.y];
   else op = pack.ops[blockIdx.y];
+#if RRL_LAT_PIN
+  {  // the pointers used after the wait held in registers from here on (not re-read from the bank)
+    const void *a = op.in1, *b = op.in2, *c1 = op.cum1, *c2 = op.cum2, *si = op.scale_in;
+    void *o = op.out, *so = op.scale_out;
+    asm volatile("" : "+l"(a), "+l"(b), "+l"(c1), "+l"(c2), "+l"(si), "+l"(o), "+l"(so));
+    op.in1 = a; op.in2 = b; op.out = o;
+    op.cum1 = static_cast<const int32_t *>(c1); op.cum2 = static_cast<const int32_t *>(c2);
+    op.scale_in = static_cast<const int32_t *>(si); op.scale_out = static_cast<int32_t *>(so);
+  }
+#endif
   const bool tip1 = op.flags & OP_TIP1, tip2 = op.flags & OP_TIP2;
   const int cat = threadIdx.x % C;  // kLatThreads is a multiple of C
   const T *__restrict__ P1g = static_cast<const T *>(op.P1) + cat * 16;
@@ -303,6 +326,10 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 #ifdef RRL_LAT_TRACE
   const unsigned long long t_entry = gtime();
   unsigned long long t_ld = 0;
+  // slot claimed at entry (its round trip overlaps the prologue), per-SM counter
+  unsigned tr_smid, tr_k = kLatSlots;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(tr_smid));
+  if (threadIdx.x == 0 && tr_smid < 160) tr_k = atomicAdd(&g_lat_n[tr_smid], 1u);
 #endif
 
   // fp32: each thread holds its category's rows in registers.  fp64: the rows
@@ -400,8 +427,8 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 #pragma unroll
         for (int z = 0; z < 4; ++z) L2[j][z] = T(0);
       }
-      ca[j] = (scale_w && valid && cat == 0 && op.cum1 != nullptr) ? __ldg(op.cum1 + pat) : 0;
-      cb[j] = (scale_w && valid && cat == 0 && op.cum2 != nullptr) ? __ldg(op.cum2 + pat) : 0;
+      ca[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum1 != nullptr) ? __ldg(op.cum1 + pat) : 0;
+      cb[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum2 != nullptr) ? __ldg(op.cum2 + pat) : 0;
     }
     if constexpr (!kRegP) {
       if (!tables) {  // block-uniform, first chunk only
@@ -428,16 +455,18 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 #ifdef RRL_LAT_TRACE
       if (j == 0 && threadIdx.x == 0 && t_ld == 0) t_ld = gtime_after((float)r[0] + (float)ca[0] + (float)cb[0]);
 #endif
+#if RRL_LAT_ABL & 2  // ablation (timing experiments only): plain store, no rescale
+      if (valid) V4<T>::st(out + (size_t)item * 4, r);
+#else
       finish_item<T, C>(op, r, valid, pat, cat, ca[j], cb[j], out + (size_t)item * 4);
+#endif
     }
   }
 #ifdef RRL_LAT_TRACE
-  __syncthreads();
+  // thread 0's stores issued (no barrier: the stamp must not delay the CTA's exit)
   if (threadIdx.x == 0) {
-    unsigned smid;
-    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    const unsigned smid = tr_smid, k = tr_k;
     const unsigned long long t_end = gtime();
-    const unsigned k = smid < 160 ? atomicAdd(&g_lat_n[smid], 1u) : kLatSlots;
     if (k < kLatSlots) {
       const unsigned long long q = smid * kLatSlots + k;
       const DevOp &op0 = INL ? pack.inl[0] : pack.ops[0];  // identifies the level set
@@ -975,6 +1004,9 @@ int launch_latency_u(const DevOp *d_ops, const DevOp *h_ops, int nops, int p, in
     at[0].val.programmaticStreamSerializationAllowed = 1;
     cfg.attrs = at;
     cfg.numAttrs = 1;
+#ifdef RRL_LAT_NO_PRETIP
+    early &= ~1;
+#endif
     cudaError_t e = pack.n <= kInline ? cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U, true>, pack, p, nchunks, early)
                                       : cudaLaunchKernelEx(&cfg, k_partials_nuc<T, C, U, false>, pack, p, nchunks, early);
     if (e != cudaSuccess) return (int)e;

@@ -3,7 +3,7 @@
 
 Builds a trace variant of the library (-DRRL_LAT_TRACE, _lib/librrl-lattrace.so):
 every CTA stamps %globaltimer at entry, after griddepcontrol.wait and at its
-end (after a closing __syncthreads).  Runs configs[1] (or another config) as
+end (thread 0, after its stores are issued; the record slot is claimed at entry).  Runs configs[1] (or another config) as
 the bench does (CUDA graph, PDL, L2 flushed before every pass) and prints,
 per level set, where the time goes:
 
