@@ -953,7 +953,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
           e = (int)cudaErrorNotSupported;
           if (tc && I->tmaps_ok)  // TMA-fed tcgen05, one CTA per tile (c <= 4)
             e = launch_update_partials_codon_tc5(I->c, I->d_ops + o0, I->h_ops + o0, nr, pmax, I->p_pad,
-                                                 &I->tmap_partials, &I->tmap_P, &I->tmap_Plo, I->stream);
+                                                 &I->tmap_partials, &I->tmap_P, &I->tmap_Plo, I->d_PT, I->stream);
           if (e == (int)cudaErrorNotSupported && tc)
             e = launch_update_partials_codon_tc(I->c, I->d_ops + o0, nr, pmax, I->p_pad, I->stream);
           if (e == (int)cudaErrorNotSupported && I->prec == 64 && !(I->flags & RRL_FLAG_CODON_SIMT))

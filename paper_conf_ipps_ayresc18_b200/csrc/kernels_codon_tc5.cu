@@ -44,7 +44,7 @@
 namespace rrl {
 
 #ifdef RRL_TC5_TRACE  // dev build only (tools/trace_tc5.py): clock64 timeline of CTA 0
-__device__ long long g_tc5_trace[12][4096];
+__device__ long long g_tc5_trace[16][4096];
 __device__ int g_tc5_kind[4096];
 #define TR(ev, g)                                                            \
   do {                                                                       \
@@ -69,11 +69,14 @@ constexpr int kThr = 15 * 32;
 // 16 KB K-halves each), one tile of lo parts, a ring of two matrix tiles (per
 // K-half h: [P hi rows 0-63 | P lo rows 0-63], 16 KB, so one N = 128 MMA reads
 // A hi once for hi.hi and hi.lo), the output staging tile.
+#ifndef RRL_TC5_ALO_TMEM
+#define RRL_TC5_ALO_TMEM 1
+#endif
 #ifndef RRL_TC5_NLO
 #define RRL_TC5_NLO 1
 #endif
 #ifndef RRL_TC5_NB
-#define RRL_TC5_NB 2
+#define RRL_TC5_NB (RRL_TC5_TIP_PT ? 2 : 3)
 #endif
 // Build knobs, all measured on configs[3] fp32 (updatePartials per pass):
 //  * RRL_TC5_DIRECT_STORE=1: write-back by direct 16-byte stores from the
@@ -89,17 +92,66 @@ constexpr int kThr = 15 * 32;
 // at ~1,350 cycles (24 tf32 MMAs) and a child tile's TMA load from HBM at
 // ~2.5 K cycles; the period stays ~2.4 K cycles per phase whichever ring
 // is deepened.
+// Round 2 (configs[3] updatePartials per pass, interleaved A/B): A_lo in TMEM
+// (RRL_TC5_ALO_TMEM) 1.535 -> 1.501 ms; the previous tile's write-back after
+// the accumulators are released (RRL_TC5_LATE_DRAIN) -> 1.458; a third matrix
+// slot (RRL_TC5_NB=3, the MMA issuer's longest wait was its P tile) -> 1.431.
+// No gain: the lo hand-over per K-half (RRL_TC5_LOSPLIT, 1.550 / 1.530 with
+// smem / TMEM lo), two TMEM lo slots with the last category kept in registers
+// (RRL_TC5_NLO=2, 1.475-1.518), tip columns from P^T (RRL_TC5_TIP_PT, 1.734).
+// RRL_TC5_LOSPLIT=1: the lo tile is handed over per K-half (two full / empty
+// barrier pairs per lo slot): the MMAs of K-half 0 start once the converters
+// finished that half, and the converters start the next phase's K-half 0 as
+// soon as this phase's K-half-0 MMAs completed (the phase chain was converter
+// then MMAs, serial, ~1.1 K + 1.3 K cycles).
+#ifndef RRL_TC5_LOSPLIT
+#define RRL_TC5_LOSPLIT 0
+#endif
+constexpr int LOH = RRL_TC5_LOSPLIT ? 2 : 1;  // lo hand-over parts per slot
+#ifndef RRL_TC5_LATE_DRAIN
+#define RRL_TC5_LATE_DRAIN 1
+#endif
 #ifndef RRL_TC5_DIRECT_STORE
 #define RRL_TC5_DIRECT_STORE 0
 #endif
+// RRL_TC5_ALO_TMEM=1: the converters write the child's tf32 lo parts into TMEM
+// (tcgen05.st, one 64-column slot) and the A_lo.P_hi MMAs read A from TMEM, so
+// the lo tile never passes through shared memory (its write and its MMA reads,
+// 64 KB of shared-memory traffic per phase, and 32 KB of ring space given to a
+// fourth child tile); K-half 1 runs as N = 128 MMAs A_hi.[P_lo | P_hi] into
+// [corr | main_1] after its first K-step (the matrix producer lands K-half 1
+// of an internal phase's P tile as [lo | hi]), so A_hi is read 9 instead of 12
+// times per phase.
+constexpr bool kAloTmem = RRL_TC5_ALO_TMEM != 0;
+// RRL_TC5_TIP_PT=1: a tip child's column P[.][obs] comes from K1's P^T slab in
+// global memory (row obs = column obs of P, row 61 = row sums), copied into a
+// per-thread shared-memory slot (cp.async) one phase ahead, so tip phases take
+// no matrix-ring slot, no TMA and no shared-memory gather.  Measured slower:
+// 1.734 vs 1.431 ms per configs[3] pass (the slot costs a child tile of the
+// ring; round 1 saw global P^T gathers lose too).  Off.
+#ifndef RRL_TC5_TIP_PT
+#define RRL_TC5_TIP_PT 0
+#endif
+constexpr bool kTipPT = RRL_TC5_TIP_PT != 0;
+
 constexpr int NLO = RRL_TC5_NLO;  // lo tiles (2: the converters run under the previous phase's MMAs)
 constexpr int NB = RRL_TC5_NB;    // matrix tiles (3: a tip phase's P tile lands while the previous one is read)
-constexpr int NA = (RRL_TC5_DIRECT_STORE ? 7 : 6) - NLO - NB;  // child tiles: 7 x 32 KB of rings fit 227 KB
-constexpr int SM_A = 0, SM_ALO = NA * 32768, SM_B = SM_ALO + NLO * 32768, SM_S1 = SM_B + NB * 32768;
-static_assert(NA >= 1 && 2 * (NA + NB + NLO) + 2 <= 16, "ring sizes / mbarrier slots");
+constexpr int NLO_SM = kAloTmem ? 0 : NLO;                          // lo tiles in shared memory
+constexpr int NPF = kTipPT ? 1 : 0;  // 32 KB: the epilogue threads' prefetched tip columns
+constexpr int NA = (RRL_TC5_DIRECT_STORE ? 7 : 6) - NLO_SM - NB - NPF;  // child tiles: 7 x 32 KB of rings fit 227 KB
+constexpr int SM_A = 0, SM_ALO = NA * 32768, SM_B = SM_ALO + NLO_SM * 32768, SM_PF = SM_B + NB * 32768,
+              SM_S1 = SM_PF + NPF * 32768;
+// Two TMEM lo slots (the converters write phase g+1's lo parts while phase g's
+// MMAs read phase g's): the budget (512 columns) then holds only C - 1 parked
+// products, so the tile's last category is written back from registers at the
+// tile's end instead of being parked.
+constexpr bool kLastInRegs = kAloTmem && NLO == 2;
+static_assert(!kAloTmem || NLO <= 2, "TMEM lo slots");
+constexpr int kBars = 24;
+static_assert(NA >= 1 && 2 * (NA + NB + NLO * LOH) + 2 <= kBars, "ring sizes / mbarrier slots");
 constexpr int SMEM_MX = SM_S1 + (RRL_TC5_DIRECT_STORE ? 0 : TM * TS * 4);  // row maxima / scale [2][128]
-constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // 16 mbarriers
-constexpr int SMEM_TMEM = SMEM_BAR + 16 * 8;
+constexpr int SMEM_BAR = SMEM_MX + 2 * TM * 4;         // kBars mbarriers
+constexpr int SMEM_TMEM = SMEM_BAR + kBars * 8;
 constexpr int SMEM_TOTAL = SMEM_TMEM + 16;
 #ifndef RRL_TC5_ACC4
 #define RRL_TC5_ACC4 0
@@ -109,7 +161,9 @@ constexpr int kTmemCols = 512;
 // N = 128 MMA A_hi.[P_hi|P_lo] + one N = 64 A_lo.P_hi), else [main_0 | corr |
 // main_1] (3 x 64: K-half 1 as three N = 64 MMAs); then one 64-column slot per
 // category (the unscaled product)
-constexpr int kProdCol = (RRL_TC5_ACC4 ? 4 : 3) * TS;
+constexpr int kAloCol = (RRL_TC5_ACC4 ? 4 : 3) * TS;     // TMEM lo slot (kAloTmem)
+constexpr int kProdCol = kAloCol + (kAloTmem ? NLO * TS : 0);
+static_assert(!(kAloTmem && RRL_TC5_ACC4), "ALO_TMEM uses the 3-accumulator layout");
 
 __device__ inline uint32_t sa(const void *p) { return static_cast<uint32_t>(__cvta_generic_to_shared(p)); }
 __device__ inline uint64_t desc_sw128(uint32_t saddr) {  // K-major, 128-byte swizzle, 8-row atoms of 1 KB
@@ -125,6 +179,12 @@ __device__ inline void mma_tf32(uint32_t d, uint64_t a, uint64_t b, uint32_t ide
       "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
       "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n}\n" ::"r"(d),
       "l"(a), "l"(b), "r"(idesc), "r"(acc));
+}
+__device__ inline void mma_tf32_ts(uint32_t d, uint32_t a_tmem, uint64_t b, uint32_t idesc, uint32_t acc) {
+  asm volatile(
+      "{\n.reg .pred p;\nsetp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n}\n" ::"r"(d),
+      "r"(a_tmem), "l"(b), "r"(idesc), "r"(acc));
 }
 __device__ inline void commit(uint64_t *bar) {
   asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(sa(bar))
@@ -181,6 +241,20 @@ __device__ inline void tmem_st16(uint32_t taddr, const float *v) {
       "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])), "r"(__float_as_uint(v[14])), "r"(__float_as_uint(v[15]))
       : "memory");
 }
+__device__ inline void tmem_st32(uint32_t taddr, const float *v) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16,"
+      "%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(taddr),
+      "r"(__float_as_uint(v[0])), "r"(__float_as_uint(v[1])), "r"(__float_as_uint(v[2])), "r"(__float_as_uint(v[3])),
+      "r"(__float_as_uint(v[4])), "r"(__float_as_uint(v[5])), "r"(__float_as_uint(v[6])), "r"(__float_as_uint(v[7])),
+      "r"(__float_as_uint(v[8])), "r"(__float_as_uint(v[9])), "r"(__float_as_uint(v[10])), "r"(__float_as_uint(v[11])),
+      "r"(__float_as_uint(v[12])), "r"(__float_as_uint(v[13])), "r"(__float_as_uint(v[14])), "r"(__float_as_uint(v[15])),
+      "r"(__float_as_uint(v[16])), "r"(__float_as_uint(v[17])), "r"(__float_as_uint(v[18])), "r"(__float_as_uint(v[19])),
+      "r"(__float_as_uint(v[20])), "r"(__float_as_uint(v[21])), "r"(__float_as_uint(v[22])), "r"(__float_as_uint(v[23])),
+      "r"(__float_as_uint(v[24])), "r"(__float_as_uint(v[25])), "r"(__float_as_uint(v[26])), "r"(__float_as_uint(v[27])),
+      "r"(__float_as_uint(v[28])), "r"(__float_as_uint(v[29])), "r"(__float_as_uint(v[30])), "r"(__float_as_uint(v[31]))
+      : "memory");
+}
 __device__ inline void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
 __device__ inline void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 __device__ inline void fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -205,16 +279,16 @@ template <int C>
 __global__ void __launch_bounds__(kThr, 1)
 k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p_pad,
                      const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmP,
-                     const __grid_constant__ CUtensorMap tmPlo) {
-  static_assert(kProdCol + C * TS <= kTmemCols, "category slots must fit TMEM");
+                     const __grid_constant__ CUtensorMap tmPlo, const float *__restrict__ PT) {
+  static_assert(kProdCol + (C - (kLastInRegs ? 1 : 0)) * TS <= kTmemCols, "category slots must fit TMEM");
   extern __shared__ __align__(1024) unsigned char sm[];
   uint64_t *a_full = reinterpret_cast<uint64_t *>(sm + SMEM_BAR);  // [NA] child tile landed
   uint64_t *a_empty = a_full + NA;                                  // [NA] its MMAs completed
   uint64_t *b_full = a_full + 2 * NA;                               // [NB] matrix tile landed
   uint64_t *b_empty = b_full + NB;                                  // [NB] MMAs / tip gather done
-  uint64_t *lo_full = b_full + 2 * NB;                              // [NLO] converters wrote the lo tile
-  uint64_t *lo_empty = lo_full + NLO;                               // [NLO] its MMAs completed
-  uint64_t *acc_full = lo_full + 2 * NLO;
+  uint64_t *lo_full = b_full + 2 * NB;                              // [NLO][LOH] converters wrote the lo tile (part)
+  uint64_t *lo_empty = lo_full + NLO * LOH;                         // [NLO][LOH] its MMAs completed
+  uint64_t *acc_full = lo_full + 2 * NLO * LOH;
   uint64_t *acc_empty = acc_full + 1;
   uint32_t *tmem_slot = reinterpret_cast<uint32_t *>(sm + SMEM_TMEM);
   float *S1 = reinterpret_cast<float *>(sm + SM_S1);
@@ -237,7 +311,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       bar_init(&b_full[i], 1);
       bar_init(&b_empty[i], 1);
     }
-    for (int i = 0; i < NLO; ++i) {
+    for (int i = 0; i < NLO * LOH; ++i) {
       bar_init(&lo_full[i], kConvThr / 32);
       bar_init(&lo_empty[i], 1);
     }
@@ -297,6 +371,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         const DevOp &op = phase_op(g, c, b, p0);
         if (p0 >= op.p) continue;
         const bool tip = is_tip(op, b);
+        if (kTipPT && tip) continue;  // the epilogue reads the column from P^T
         const uint32_t sl = gb % NB, use = gb / NB;
         ++gb;
         bar_wait(&b_empty[sl], (use & 1u) ^ 1u);
@@ -306,11 +381,14 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         const uint32_t dst = sbase + SM_B + sl * 32768;
         const int mat = b == 0 ? op.mat1 : op.mat2;
         bar_expect(&b_full[sl], tip ? 16384u : 32768u);
+        // K-half h at h * 16 KB: [P hi | P lo] (8 KB each); K-half 1 of an internal phase
+        // as [P lo | P hi] with ALO_TMEM (its N = 128 MMAs write [corr | main_1])
+        const uint32_t h1hi = (!tip && kAloTmem) ? 8192u : 0u;
         tma4(dst, &tmP, 0, 0, c, mat, &b_full[sl]);
-        tma4(dst + 16384, &tmP, 32, 0, c, mat, &b_full[sl]);
+        tma4(dst + 16384 + h1hi, &tmP, 32, 0, c, mat, &b_full[sl]);
         if (!tip) {  // the matrix's tf32 low parts, precomputed by K1
           tma4(dst + 8192, &tmPlo, 0, 0, c, mat, &b_full[sl]);
-          tma4(dst + 16384 + 8192, &tmPlo, 32, 0, c, mat, &b_full[sl]);
+          tma4(dst + 16384 + (8192u - h1hi), &tmPlo, 32, 0, c, mat, &b_full[sl]);
         }
       }
     }
@@ -323,15 +401,20 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         int c, b, p0;
         const DevOp &op = phase_op(g, c, b, p0);
         if (p0 >= op.p) continue;
+        if (kTipPT && is_tip(op, b)) continue;  // no matrix slot, no MMA
         const uint32_t bs = gb % NB;
         bar_wait(&b_full[bs], (uint32_t)(gb / NB) & 1u);
+        TR(12, g);
         ++gb;
         if (is_tip(op, b)) continue;  // a tip child is a P-column gather in the epilogue: no MMA
         const uint32_t sl = ia % NA, use = ia / NA;
         bar_wait(&a_full[sl], use & 1u);
-        const uint32_t ls = ia % NLO;
-        bar_wait(&lo_full[ls], (ia / NLO) & 1u);
+        TR(13, g);
+        const uint32_t ls = ia % NLO, lpar = (ia / NLO) & 1u;
+        if (LOH == 1) bar_wait(&lo_full[ls], lpar);
+        TR(14, g);
         bar_wait(acc_empty, (ia & 1u) ^ 1u);  // the epilogue drained the previous accumulators
+        TR(15, g);
         ++ia;
         fence_after();
         TR(3, g);
@@ -346,10 +429,29 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
 #pragma unroll
         for (int kk = 0; kk < TS / 8; ++kk) {
           const int h = kk >> 2, kin = kk & 3;
+          if (LOH == 2 && kin == 0) {  // this K-half's lo part written by the converters
+            bar_wait(&lo_full[ls * LOH + h], lpar);
+            fence_after();
+          }
           const uint64_t ah = desc_sw128(sbase + SM_A + sl * 32768 + h * 16384 + kin * 32);
           const uint64_t al = desc_sw128(sbase + SM_ALO + ls * 32768 + h * 16384 + kin * 32);
           const uint64_t bb = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + kin * 32);
-          if (RRL_TC5_ACC4) {
+          if (kAloTmem) {
+            const uint32_t at = tmem + (uint32_t)(kAloCol + ls * TS + kk * 8);  // A_lo columns of this K-step
+            if (h == 0) {  // B = [P hi | P lo]
+              mma_tf32(tmem, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);  // [main_0 | corr]
+              mma_tf32_ts(tmem + TS, at, bb, idesc_tf32(TS), 1u);             // corr += A_lo P_hi
+            } else {       // B = [P lo | P hi]
+              const uint64_t bh = desc_sw128(sbase + SM_B + bs * 32768 + h * 16384 + 8192 + kin * 32);
+              if (kin == 0) {  // main_1 starts here, corr accumulates: two N = 64
+                mma_tf32(tmem + 2 * TS, ah, bh, idesc_tf32(TS), 0u);
+                mma_tf32(tmem + TS, ah, bb, idesc_tf32(TS), 1u);
+              } else {
+                mma_tf32(tmem + TS, ah, bb, idesc_tf32(2 * TS), 1u);  // [corr | main_1]
+              }
+              mma_tf32_ts(tmem + TS, at, bh, idesc_tf32(TS), 1u);
+            }
+          } else if (RRL_TC5_ACC4) {
             const uint32_t d = tmem + (uint32_t)(h * 2 * TS);
             mma_tf32(d, ah, bb, idesc_tf32(2 * TS), kin > 0 ? 1u : 0u);  // [main_h | corr_h]
             mma_tf32(d + TS, al, bb, idesc_tf32(TS), 1u);                // corr_h += A_lo P_hi
@@ -362,9 +464,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
             mma_tf32(tmem + TS, ah, bl, idesc_tf32(TS), 1u);
             mma_tf32(tmem + TS, al, bb, idesc_tf32(TS), 1u);
           }
+          if (LOH == 2 && kin == 3) commit(&lo_empty[ls * LOH + h]);  // this K-half's lo part is free
         }
         commit(&a_empty[sl]);  // child tile, lo tile and matrix tile free once these MMAs completed
-        commit(&lo_empty[ls]);
+        if (LOH == 1) commit(&lo_empty[ls]);
         commit(&b_empty[bs]);
         commit(acc_full);  // accumulators ready for the epilogue
         TR(4, g);
@@ -380,14 +483,51 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       if (is_tip(op, b) || p0 >= op.p) continue;
       const uint32_t sl = ia % NA, use = ia / NA;
       bar_wait(&a_full[sl], use & 1u);
-      const uint32_t ls = ia % NLO;
-      bar_wait(&lo_empty[ls], ((ia / NLO) & 1u) ^ 1u);  // the MMAs NLO internal phases back read this lo tile
+      const uint32_t ls = ia % NLO, lpar = ((ia / NLO) & 1u) ^ 1u;
       ++ia;
-      if (ct == 0) TR(1, g);
       const unsigned char *src = sm + SM_A + sl * 32768;
       unsigned char *dst = sm + SM_ALO + ls * 32768;
+      if constexpr (kAloTmem) {
+        // thread = tile row (TMEM lane) r of this warp's lane quarter; per K-half its 8
+        // swizzled 16-byte chunks (states 4j..4j+3 at chunk j ^ (r & 7)) -> 32 lo parts
+        // -> TMEM columns kAloCol + 32 h + (0..31)
+        const int wq = warp & 3, r = wq * 32 + lane;
+        const uint32_t trow = tmem + ((uint32_t)(wq * 32) << 16) + (uint32_t)(kAloCol + ls * TS);
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          if (h == 0 || LOH == 2) {  // the MMAs of the previous internal phase read this slot (part)
+            bar_wait(&lo_empty[ls * LOH + (LOH == 2 ? h : 0)], lpar);
+            fence_after();
+            if (ct == 0 && h == 0) TR(1, g);
+          }
+          float lo[32];
+#pragma unroll
+          for (int j = 0; j < 8; ++j) {
+            const float4 v = *reinterpret_cast<const float4 *>(src + h * 16384 + r * 128 + ((j ^ (r & 7)) << 4));
+            lo[4 * j] = lo_tf32(v.x);
+            lo[4 * j + 1] = lo_tf32(v.y);
+            lo[4 * j + 2] = lo_tf32(v.z);
+            lo[4 * j + 3] = lo_tf32(v.w);
+          }
+          tmem_st32(trow + (uint32_t)(h * 32), lo);
+          if (LOH == 2 || h == 1) {
+            tmem_wait_st();
+            fence_before();
+            __syncwarp();
+            if (lane == 0) bar_arrive(&lo_full[ls * LOH + (LOH == 2 ? h : 0)]);
+          }
+        }
+        if (ct == 0) TR(2, g);
+        continue;
+      }
+      // chunk u * kConvThr + ct of the 2,048 16-byte chunks: u < 8 is K-half 0, u >= 8 K-half 1
 #pragma unroll
       for (int u = 0; u < TM * 16 / kConvThr; u += 8) {  // lo of every 16-byte chunk, same swizzled offset
+        const int part = LOH == 2 ? u / 8 : 0;
+        if (u == 0 || LOH == 2) {  // the MMAs NLO internal phases back read this lo tile (part)
+          bar_wait(&lo_empty[ls * LOH + part], lpar);
+          if (ct == 0 && u == 0) TR(1, g);
+        }
         float4 v[8];
 #pragma unroll
         for (int q = 0; q < 8; ++q) v[q] = *reinterpret_cast<const float4 *>(src + (ct + (u + q) * kConvThr) * 16);
@@ -395,11 +535,13 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         for (int q = 0; q < 8; ++q)
           *reinterpret_cast<float4 *>(dst + (ct + (u + q) * kConvThr) * 16) =
               make_float4(lo_tf32(v[q].x), lo_tf32(v[q].y), lo_tf32(v[q].z), lo_tf32(v[q].w));
+        if (LOH == 2 || u + 8 >= TM * 16 / kConvThr) {
+          asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
+          __syncwarp();
+          if (lane == 0) bar_arrive(&lo_full[ls * LOH + part]);
+        }
       }
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> async proxy
-      __syncwarp();
       if (ct == 0) TR(2, g);
-      if (lane == 0) bar_arrive(&lo_full[ls]);
     }
   } else {
     // ================================================================ epilogue
@@ -438,31 +580,23 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
     int prev_y = 0, prev_buf = 0;
     float *prev_dst = nullptr;  // direct write-back: row p0 of category 0 of the previous tile's output
     bool have_prev = false;
-    auto drain = [&](int cat) {
-      float w0[16], w1[16];
-      tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), w0);
-      tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), w1);
-      tmem_wait_ld();
+    // scale the 32 values of this thread's row half of category `cat` of the
+    // previous tile by 2^-e, stage them, and hand the tile to a TMA store
+    auto stage_store = [&](int cat, const float (&w)[32]) {
       if (RRL_TC5_DIRECT_STORE) {
         float4 *dst = reinterpret_cast<float4 *>(prev_dst + ((size_t)cat * p_pad + r) * TS + h * 32);
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          dst[k] = make_float4(w0[4 * k] * sc_prev, w0[4 * k + 1] * sc_prev, w0[4 * k + 2] * sc_prev,
-                               w0[4 * k + 3] * sc_prev);
-          dst[4 + k] = make_float4(w1[4 * k] * sc_prev, w1[4 * k + 1] * sc_prev, w1[4 * k + 2] * sc_prev,
-                                   w1[4 * k + 3] * sc_prev);
-        }
+        for (int k = 0; k < 8; ++k)
+          dst[k] = make_float4(w[4 * k] * sc_prev, w[4 * k + 1] * sc_prev, w[4 * k + 2] * sc_prev,
+                               w[4 * k + 3] * sc_prev);
         return;
       }
       if (tid == 0) bulk_wait_read0();  // the previous store has read the staging tile
       named_sync(1, kEpiThr);
 #pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        *s1(r, h, k) = make_float4(w0[4 * k] * sc_prev, w0[4 * k + 1] * sc_prev, w0[4 * k + 2] * sc_prev,
-                                   w0[4 * k + 3] * sc_prev);
-        *s1(r, h, 4 + k) = make_float4(w1[4 * k] * sc_prev, w1[4 * k + 1] * sc_prev, w1[4 * k + 2] * sc_prev,
-                                       w1[4 * k + 3] * sc_prev);
-      }
+      for (int k = 0; k < 8; ++k)
+        *s1(r, h, k) = make_float4(w[4 * k] * sc_prev, w[4 * k + 1] * sc_prev, w[4 * k + 2] * sc_prev,
+                                   w[4 * k + 3] * sc_prev);
       asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> TMA store
       named_sync(1, kEpiThr);
       if (tid == 0) {
@@ -470,6 +604,36 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         tma_store4(&tmA, 32, prev_y, cat, prev_buf, sa(S1) + TM * 128);
         bulk_commit();
       }
+    };
+    auto drain = [&](int cat) {  // a parked category of the previous tile
+      float w[32];
+      tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS), *reinterpret_cast<float(*)[16]>(w));
+      tmem_ld16(tl + (uint32_t)(kProdCol + cat * TS + 16), *reinterpret_cast<float(*)[16]>(w + 16));
+      tmem_wait_ld();
+      stage_store(cat, w);
+    };
+    constexpr int kParked = C - (kLastInRegs ? 1 : 0);  // categories written back during the next tile
+    // tip column of the next phase (kTipPT): 128 bytes of P^T copied by cp.async
+    // into this thread's slot one phase ahead ([k][thread] float4 layout: a warp's
+    // k-th float4s are 512 contiguous bytes)
+    const uint32_t pf_s = sbase + SM_PF + (uint32_t)tid * 16;
+    int lt_cur = 0;
+    auto issue_pf = [&](int g2) {
+      if (!kTipPT || g2 >= nphase) return;
+      const int lt2 = g2 / (2 * C), c2 = (g2 / 2) % C, b2 = g2 & 1;
+      const int f2 = blockIdx.x + lt2 * gridDim.x;
+      const DevOp &op2 = ops[f2 / ntiles];
+      if (!(op2.flags & (b2 == 0 ? OP_TIP1 : OP_TIP2)) || (f2 % ntiles) * TM >= op2.p) return;
+      const uint32_t svw = lt2 == lt_cur ? sv_cur : sv_nxt;
+      unsigned sv = (svw >> (8 * b2)) & 0xffu;
+      sv = sv < (unsigned)kS61 ? sv : (unsigned)kS61;  // row 61 = row sums (missing state)
+      const float *src = PT + ((size_t)(b2 == 0 ? op2.mat1 : op2.mat2) * C + c2) * (TS * TS) + sv * TS + h * 32;
+#pragma unroll
+      for (int k = 0; k < 8; ++k)
+        asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(pf_s + (uint32_t)(k * kEpiThr * 16)),
+                     "l"(src + 4 * k)
+                     : "memory");
+      asm volatile("cp.async.commit_group;" ::: "memory");
     };
     float m = 0.f;  // running max over (c, z) of this thread's row half
     float d1[32];     // child 1's contraction of the current category
@@ -486,16 +650,37 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         if (lt == 0) load_meta(0, sv_nxt, ex_nxt);
         sv_cur = sv_nxt;
         ex_cur = ex_nxt;
+        lt_cur = lt;
         if (lt + 1 < my_tiles) load_meta(lt + 1, sv_nxt, ex_nxt);
+        if (lt == 0) issue_pf(0);
       }
+      const bool tip_ph = (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) != 0;
+      float dv[32];
+      if (kTipPT && tip_ph) {  // this phase's column, copied during the previous phase
+        asm volatile("cp.async.wait_group 0;" ::: "memory");
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const float4 v = *reinterpret_cast<const float4 *>(sm + SM_PF + (k * kEpiThr + tid) * 16);
+          dv[4 * k] = v.x;
+          dv[4 * k + 1] = v.y;
+          dv[4 * k + 2] = v.z;
+          dv[4 * k + 3] = v.w;
+        }
+      }
+      issue_pf(g + 1);
       if (p0 >= op.p) continue;  // past this op's own range (a shorter partition): another op's rows
-      const uint32_t gcur = gb++;
-      if (b == 0 && have_prev) {  // before child 1 reuses slot c: write back the previous tile's category c
+      const uint32_t gcur = (kTipPT && tip_ph) ? 0u : gb++;
+      // Write-back of the previous tile's category c (slot c is reused by this tile's
+      // product of category c): RRL_TC5_LATE_DRAIN=1 after this phase's accumulators
+      // are read and released, so the staging / TMA-store round trip is off the MMAs' path.
+      if (!RRL_TC5_LATE_DRAIN && b == 0 && have_prev && c < kParked) {
         drain(c);
         if (tid == 0) TR(9, g);
       }
-      float dv[32];
-      if (op.flags & (b == 0 ? OP_TIP1 : OP_TIP2)) {
+      if (kTipPT && tip_ph) {
+        if (tid == 0) TR(7, g);
+        if (tid == 0) TR(5, g);
+      } else if (tip_ph) {
         // Tip child: sum_x P[z][x] [x == obs] = P[z][obs], read from the raw fp32 P tile the
         // producer landed in stage g&1 (swizzled K-major: row z, 16-byte chunk (x&31)/4 at
         // position chunk ^ (z&7) of half x>>5). A missing state (code >= 61) is the row sum.
@@ -562,6 +747,10 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       if (b == 0) {  // child 1 waits in registers: child 2's phase of the same category is next
 #pragma unroll
         for (int i = 0; i < 32; ++i) d1[i] = dv[i];
+        if (RRL_TC5_LATE_DRAIN && have_prev && c < kParked) {
+          drain(c);
+          if (tid == 0) TR(9, g);
+        }
         if (tid == 0) TR(6, g);
         continue;
       }
@@ -570,9 +759,11 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         dv[i] *= d1[i];
         m = fmaxf(m, dv[i]);
       }
-      tmem_st16(slot, dv);  // park the unscaled product (in place of child 1) until written back
-      tmem_st16(slot + 16, dv + 16);
-      tmem_wait_st();
+      if (c < kParked) {
+        tmem_st16(slot, dv);  // park the unscaled product until written back
+        tmem_st16(slot + 16, dv + 16);
+        tmem_wait_st();
+      }
       if (c < C - 1) {
         if (tid == 0) TR(6, g);
         continue;
@@ -600,11 +791,12 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
       prev_buf = op.bufd;
       prev_dst = static_cast<float *>(op.out) + (size_t)p0 * TS;
       have_prev = true;
+      if (kLastInRegs) stage_store(C - 1, dv);  // the last category, straight from registers
       if (tid == 0) TR(6, g);
       m = 0.f;
     }
     if (have_prev)  // the CTA's last tile
-      for (int cat = 0; cat < C; ++cat) drain(cat);
+      for (int cat = 0; cat < kParked; ++cat) drain(cat);
   }
   if (tid == 0) bulk_wait0();  // output stores complete before the grid does
   fence_before();
@@ -614,7 +806,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
 
 template <int C>
 int launch_tc5(const DevOp *d_ops, int nops, int p, int p_pad, const CUtensorMap *tA, const CUtensorMap *tP,
-               const CUtensorMap *tPlo, cudaStream_t st) {
+               const CUtensorMap *tPlo, const float *PT, cudaStream_t st) {
   static int nsm_dev[kMaxDevices] = {};
   int &nsm = nsm_dev[device_slot()];
   if (nsm == 0) {
@@ -640,14 +832,14 @@ int launch_tc5(const DevOp *d_ops, int nops, int p, int p_pad, const CUtensorMap
   cfg.attrs = at;
   cfg.numAttrs = 1;
   return (int)cudaLaunchKernelEx(&cfg, k_partials_codon_tc5<C>, d_ops, ntiles, (int)total, p_pad, *tA, *tP,
-                                 *tPlo);
+                                 *tPlo, PT);
 }
 
 }  // namespace
 
 int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
                                      int p_pad, const void *tmap_partials, const void *tmap_P,
-                                     const void *tmap_Plo, void *stream) {
+                                     const void *tmap_Plo, const void *d_PT, void *stream) {
   // every child must live in the tensor-mapped slab (internal buffers) or be tip states; the
   // destination is always in the slab (its tile is written back by TMA store)
   for (int i = 0; i < nops; ++i)
@@ -659,9 +851,9 @@ int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_o
   const CUtensorMap *tP = static_cast<const CUtensorMap *>(tmap_P);
   const CUtensorMap *tPlo = static_cast<const CUtensorMap *>(tmap_Plo);
   switch (c) {
-    case 1: return launch_tc5<1>(d_ops, nops, p, p_pad, tA, tP, tPlo, st);
-    case 2: return launch_tc5<2>(d_ops, nops, p, p_pad, tA, tP, tPlo, st);
-    case 4: return launch_tc5<4>(d_ops, nops, p, p_pad, tA, tP, tPlo, st);
+    case 1: return launch_tc5<1>(d_ops, nops, p, p_pad, tA, tP, tPlo, static_cast<const float *>(d_PT), st);
+    case 2: return launch_tc5<2>(d_ops, nops, p, p_pad, tA, tP, tPlo, static_cast<const float *>(d_PT), st);
+    case 4: return launch_tc5<4>(d_ops, nops, p, p_pad, tA, tP, tPlo, static_cast<const float *>(d_PT), st);
     default: return (int)cudaErrorNotSupported;
   }
 }
@@ -669,7 +861,7 @@ int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_o
 }  // namespace rrl
 
 #ifdef RRL_TC5_TRACE
-extern "C" int rrl_debug_tc5_trace(long long *ev /*[12*4096]*/, int *kind /*[4096]*/) {
+extern "C" int rrl_debug_tc5_trace(long long *ev /*[16*4096]*/, int *kind /*[4096]*/) {
   if (cudaMemcpyFromSymbol(ev, rrl::g_tc5_trace, sizeof(rrl::g_tc5_trace)) != cudaSuccess) return -1;
   if (cudaMemcpyFromSymbol(kind, rrl::g_tc5_kind, sizeof(rrl::g_tc5_kind)) != cudaSuccess) return -1;
   return 0;

@@ -75,7 +75,7 @@ int launch_update_partials_codon_tc(int c, const DevOp *d_ops, int nops, int p, 
 int launch_split_tf32(const float *x, float *lo, size_t n, void *stream);
 int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_ops, int nops, int p,
                                      int p_pad, const void *tmap_partials, const void *tmap_P,
-                                     const void *tmap_Plo, void *stream);
+                                     const void *tmap_Plo, const void *d_PT, void *stream);
 // fp64 codon operations on the FP64 tensor cores (mma.sync m8n8k4 f64), c in {1, 2, 4, 8}.
 int launch_update_partials_codon_dmma(int c, const DevOp *d_ops, int nops, int p, int p_pad, const void *d_PT,
                                       void *stream);

@@ -47,7 +47,7 @@ def main():
     R.rrl_update_partials(tl.inst, ops, np.array([0, b - a], np.int32))
     R.rrl_synchronize(tl.inst)
     lib = C.CDLL(LIB)
-    ev = np.zeros((12, 4096), np.int64)
+    ev = np.zeros((16, 4096), np.int64)
     kind = np.zeros(4096, np.int32)
     assert lib.rrl_debug_tc5_trace(ev.ctypes.data_as(C.c_void_p), kind.ctypes.data_as(C.c_void_p)) == 0
     ntiles = (w.p + 127) // 128
@@ -84,6 +84,28 @@ def main():
         wait_tma = ev[1, idx] - ev[0, idx]
         print(f"{lab:8s}: TMA issue->landed(conv start) {np.median(wait_tma):.0f}  conv {np.median(conv):.0f}  "
               f"MMA issue {np.median(mma) if lab == 'internal' else 0:.0f}  epilogue {np.median(epi):.0f} (median cycles)")
+    # MMA issuer: which wait released each internal phase, measured from the
+    # previous internal phase's commit (M1)
+    idx = [g for g in range(1, nph) if kind[g] == 0 and ev[3, g] > 0]
+    prev = {}
+    last = None
+    for g in range(nph):
+        if kind[g] == 0:
+            prev[g] = last
+            last = g
+    rows = []
+    for g in idx:
+        pg = prev.get(g)
+        if pg is None:
+            continue
+        base = ev[4, pg]
+        rows.append([ev[12, g] - base, ev[13, g] - base, ev[14, g] - base, ev[15, g] - base, ev[3, g] - base,
+                     ev[4, g] - ev[3, g]])
+    if rows:
+        r = np.median(np.array(rows), axis=0)
+        print("MMA issuer, cycles after the previous internal phase's commit (median): "
+              f"b_full {r[0]:.0f}  a_full {r[1]:.0f}  lo_full {r[2]:.0f}  acc_empty {r[3]:.0f}  start {r[4]:.0f}; "
+              f"issue {r[5]:.0f}")
     tl.close()
 
 
