@@ -14,7 +14,10 @@ paper; the e2e leg repeats them every step.
 `value` = effective GFLOPS of Eq. (1) (flops per pattern per pass
 (n-1) c s (4s-1), A16) summed over ranks / max-over-ranks device
 time of the K steps.  Inputs are resident in HBM; L2 (126 MB) is flushed by a
-512 MiB memset before every step, outside the per-step CUDA events.
+512 MiB memset before every step, outside the per-step CUDA events.  The K
+steps are timed with the library's profiling off; a second pass of K steps
+with it on (CUDA events around every graph replay of the updatePartials
+region) gives the region's duration for `updatePartials` and `roofline`.
 
 Multi-GPU (one process per GPU; `--gpus N` without torchrun re-launches itself
 under torch.distributed.run): the headline is weak scaling -- every rank owns
@@ -430,31 +433,42 @@ def main():
 
     def timed(tl, steps, warmup, clocks=None, fn=None):
         """Per-step CUDA events on the launching stream; L2 flushed before
-        every step outside the events; barrier + synchronize on both sides."""
+        every step outside the events; barrier + synchronize on both sides.
+        Two passes of `steps` steps: the step times come from a pass with the
+        library's profiling off (its event records between launches would sit
+        inside the timed step); the updatePartials region times (the
+        roofline's launch durations) from a second pass with it on."""
         fn = fn or step
         for _ in range(warmup):
             flush.zero_()
             fn(tl)
         barrier()
-        evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-               for _ in range(steps)]
-        # library profiling: CUDA events on this stream around every graph
-        # replay of the updatePartials region (the roofline's launch durations)
-        R.rrl_set_profiling(tl.inst, True)
-        R.rrl_reset_profile(tl.inst)
-        for i, (a, b) in enumerate(evs):
-            flush.zero_()
-            a.record(stream)
-            fn(tl)
-            b.record(stream)
-            if clocks is not None and i % 16 == 15:
-                clocks.sample()  # the GPU is still running enqueued steps
-        if clocks is not None:
-            clocks.sample()
-        barrier()
-        per = [a.elapsed_time(b) for a, b in evs]
-        prof = R.rrl_get_profile(tl.inst)
-        R.rrl_set_profiling(tl.inst, False)
+
+        def run(profile):
+            evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+                   for _ in range(steps)]
+            if profile:  # CUDA events on this stream around every graph replay of the region
+                R.rrl_set_profiling(tl.inst, True)
+                R.rrl_reset_profile(tl.inst)
+            for i, (a, b) in enumerate(evs):
+                flush.zero_()
+                a.record(stream)
+                fn(tl)
+                b.record(stream)
+                if clocks is not None and not profile and i % 16 == 15:
+                    clocks.sample()  # the GPU is still running enqueued steps
+            if clocks is not None and not profile:
+                clocks.sample()
+            barrier()
+            per = [a.elapsed_time(b) for a, b in evs]
+            prof = None
+            if profile:
+                prof = R.rrl_get_profile(tl.inst)
+                R.rrl_set_profiling(tl.inst, False)
+            return per, prof
+
+        per, _ = run(False)
+        _, prof = run(True)
         return maxall(sum(per)), prof, {"best": maxall(min(per)), "median": maxall(float(np.median(per)))}
 
     def roofline_of(cfg, precision, w, sched, part_ms, launches_per_pass):
