@@ -62,7 +62,8 @@ constexpr int kInline = RRL_LAT_INLINE;
 // 0.151; the tip-state array bulk-prefetched into L2 by the first set 0.157
 // (one SM's bulk engine streams 1.3 MB while that CTA cannot retire); 2 or 4
 // inline descriptors instead of 8 0.117 / 0.118 (the pointer path for a
-// 2-operation set: 0.147).  fp64 (tables in shared memory already) keeps 3
+// 2-operation set: 0.147); children read with ld.global.cg instead of .nc
+// (RRL_LAT_CG) 0.1174 vs 0.1173.  fp64 (tables in shared memory already) keeps 3
 // CTAs per SM: at 5 it spills and is no faster.
 #ifndef RRL_LAT_MINB
 #define RRL_LAT_MINB 12
@@ -82,6 +83,9 @@ constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 #endif
 #ifndef RRL_LAT_ABL  // timing ablations (dev builds only; results are wrong): 1 no child exponents, 2 no rescale
 #define RRL_LAT_ABL 0
+#endif
+#ifndef RRL_LAT_CG  // children and their exponents read with ld.global.cg (L2 only) instead of ld.global.nc
+#define RRL_LAT_CG 0
 #endif
 #ifndef RRL_LAT_PIN
 #define RRL_LAT_PIN 0
@@ -112,6 +116,10 @@ template <> struct V4<float> {
     const float4 x = __ldg(reinterpret_cast<const float4 *>(p));
     v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
   }
+  __device__ static inline void ldcg(const float *p, float (&v)[4]) {  // L2 only (no L1 allocation)
+    const float4 x = __ldcg(reinterpret_cast<const float4 *>(p));
+    v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
+  }
   __device__ static inline void lds(const float *p, float (&v)[4]) {
     const float4 x = *reinterpret_cast<const float4 *>(p);
     v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w;
@@ -124,6 +132,11 @@ template <> struct V4<double> {
   __device__ static inline void ld(const double *p, double (&v)[4]) {
     const double2 a = __ldg(reinterpret_cast<const double2 *>(p));
     const double2 b = __ldg(reinterpret_cast<const double2 *>(p) + 1);
+    v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
+  }
+  __device__ static inline void ldcg(const double *p, double (&v)[4]) {
+    const double2 a = __ldcg(reinterpret_cast<const double2 *>(p));
+    const double2 b = __ldcg(reinterpret_cast<const double2 *>(p) + 1);
     v[0] = a.x; v[1] = a.y; v[2] = b.x; v[3] = b.y;
   }
   __device__ static inline void lds(const double *p, double (&v)[4]) {
@@ -414,7 +427,8 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
       if (tip1) {
         s1[j] = pre ? s1p[j] : valid ? (unsigned)__ldg(S1g + pat) : 4u;
       } else if (valid) {
-        V4<T>::ld(L1g + (size_t)item * 4, L1[j]);
+        if (RRL_LAT_CG) V4<T>::ldcg(L1g + (size_t)item * 4, L1[j]);
+        else V4<T>::ld(L1g + (size_t)item * 4, L1[j]);
       } else {
 #pragma unroll
         for (int z = 0; z < 4; ++z) L1[j][z] = T(0);
@@ -422,13 +436,14 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
       if (tip2) {
         s2[j] = pre ? s2p[j] : valid ? (unsigned)__ldg(S2g + pat) : 4u;
       } else if (valid) {
-        V4<T>::ld(L2g + (size_t)item * 4, L2[j]);
+        if (RRL_LAT_CG) V4<T>::ldcg(L2g + (size_t)item * 4, L2[j]);
+        else V4<T>::ld(L2g + (size_t)item * 4, L2[j]);
       } else {
 #pragma unroll
         for (int z = 0; z < 4; ++z) L2[j][z] = T(0);
       }
-      ca[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum1 != nullptr) ? __ldg(op.cum1 + pat) : 0;
-      cb[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum2 != nullptr) ? __ldg(op.cum2 + pat) : 0;
+      ca[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum1 != nullptr) ? (RRL_LAT_CG ? __ldcg(op.cum1 + pat) : __ldg(op.cum1 + pat)) : 0;
+      cb[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum2 != nullptr) ? (RRL_LAT_CG ? __ldcg(op.cum2 + pat) : __ldg(op.cum2 + pat)) : 0;
     }
     if constexpr (!kRegP) {
       if (!tables) {  // block-uniform, first chunk only
