@@ -321,8 +321,10 @@ int rrl_create_instance(int tip_count, int partials_buffer_count, int state_coun
   I->mat_elems = (size_t)I->c * I->s_pad * I->s_pad;
   I->tip_partials.assign(tip_count, nullptr);
   I->has_states.assign(tip_count, 0);
-  // K4/K6 grid: a thread per pattern (4 states) or a warp per pattern (61 states)
-  I->nblocks = std::min(148 * 4, (pattern_count + (state_count == 61 ? 7 : 255)) / (state_count == 61 ? 8 : 256));
+  // K4/K6 grid: c threads per pattern (4 states, K4; K6 takes a thread per pattern
+  // within the same grid) or a warp per pattern (61 states)
+  I->nblocks = std::min(148 * 4, state_count == 61 ? (pattern_count + 7) / 8
+                                                   : (int)(((long long)pattern_count * category_count + 255) / 256));
   auto bail = [&](int code, const std::string &m) {
     destroy(I);
     return fail(code, m);
@@ -1072,7 +1074,7 @@ static int root_common(Instance *I, int root_buffer, int cat_weights_idx, int fr
   const int32_t *cum = cumulative_idx >= 0 ? I->d_scale + (size_t)cumulative_idx * I->p_pad + pb : nullptr;
   const size_t pel = (I->s == 4 ? (size_t)I->c * 4 : (size_t)I->s_pad) * pb * I->elt;
   const int np = pe - pb;
-  const int per_block = I->s == 61 ? 8 : 256;  // patterns per K4 block (a warp per codon pattern)
+  const int per_block = I->s == 61 ? 8 : std::max(1, 256 / I->c);  // patterns per K4 block
   const int nb = std::max(1, std::min(I->nblocks, (np + per_block - 1) / per_block));
   {
     Timed tm(I, 2);

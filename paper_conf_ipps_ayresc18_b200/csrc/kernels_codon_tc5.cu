@@ -44,7 +44,7 @@
 namespace rrl {
 
 #ifdef RRL_TC5_TRACE  // dev build only (tools/trace_tc5.py): clock64 timeline of CTA 0
-__device__ long long g_tc5_trace[16][4096];
+__device__ long long g_tc5_trace[18][4096];
 __device__ int g_tc5_kind[4096];
 #define TR(ev, g)                                                            \
   do {                                                                       \
@@ -375,6 +375,7 @@ k_partials_codon_tc5(const DevOp *__restrict__ ops, int ntiles, int total, int p
         const uint32_t sl = gb % NB, use = gb / NB;
         ++gb;
         bar_wait(&b_empty[sl], (use & 1u) ^ 1u);
+        TR(16, g);  // matrix tile issued
 #ifdef RRL_TC5_TRACE
         if (blockIdx.x == 0 && g < 4096) g_tc5_kind[g] = tip ? 1 : 0;
 #endif
@@ -861,7 +862,7 @@ int launch_update_partials_codon_tc5(int c, const DevOp *d_ops, const DevOp *h_o
 }  // namespace rrl
 
 #ifdef RRL_TC5_TRACE
-extern "C" int rrl_debug_tc5_trace(long long *ev /*[16*4096]*/, int *kind /*[4096]*/) {
+extern "C" int rrl_debug_tc5_trace(long long *ev /*[18*4096]*/, int *kind /*[4096]*/) {
   if (cudaMemcpyFromSymbol(ev, rrl::g_tc5_trace, sizeof(rrl::g_tc5_trace)) != cudaSuccess) return -1;
   if (cudaMemcpyFromSymbol(kind, rrl::g_tc5_kind, sizeof(rrl::g_tc5_kind)) != cudaSuccess) return -1;
   return 0;

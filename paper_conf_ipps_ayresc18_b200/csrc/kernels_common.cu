@@ -49,6 +49,39 @@ __global__ void k_transition(int s, int s_pad, int C, const double *__restrict__
   }
 }
 
+// K1 for 4 states: one thread per (listed matrix, category, row z), its four
+// outputs P[z][0..3] stored as one vector -- the same sums in the same order
+// as k_transition (bit-identical), without a block (and its 32 KB of shared
+// staging and barrier) per (matrix, category): configs[1] lists 254 matrices
+// x 4 categories, 1,016 blocks of 16 busy threads before.
+template <typename T>
+__global__ void __launch_bounds__(128)
+k_transition4(int C, int items, const double *__restrict__ eig, const double *__restrict__ rates,
+              const int32_t *__restrict__ idx, const double *__restrict__ tlen, T *__restrict__ P) {
+  const int t = blockIdx.x * blockDim.x + threadIdx.x;  // ((m * C) + c) * 4 + z
+  if (t >= items * C * 4) return;
+  const int z = t & 3, mc = t >> 2, m = mc / C, c = mc % C;
+  const double *V = eig, *Vi = eig + 16, *lam = eig + 32;
+  const double rt = __ldg(rates + c) * __ldg(tlen + m);
+  double ex[4], vz[4];
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    ex[k] = exp(__ldg(lam + k) * rt);
+    vz[k] = __ldg(V + z * 4 + k);
+  }
+  T o[4];
+#pragma unroll
+  for (int x = 0; x < 4; ++x) {
+    double acc = 0.0;
+#pragma unroll
+    for (int k = 0; k < 4; ++k) acc = fma(vz[k] * ex[k], __ldg(Vi + k * 4 + x), acc);
+    o[x] = (T)acc;
+  }
+  T *out = P + ((size_t)__ldg(idx + m) * C + c) * 16 + z * 4;
+#pragma unroll
+  for (int x = 0; x < 4; ++x) out[x] = o[x];
+}
+
 // K1 for the codon state space (s_pad = 64): one block per (listed matrix,
 // category).  The same sum as above, register-tiled: thread (ty, tx) of a
 // 16 x 16 block owns the 4 x 4 outputs z in [4ty, 4ty+4), x in [4tx, 4tx+4),
@@ -285,6 +318,45 @@ k_root(const T *__restrict__ L, int s, int s_pad, int C, const double *__restric
   finish_sum(part, red, blocks, count, out);
 }
 
+// K4 for 4 states: C threads per pattern, thread c reads the pattern's
+// category-c vector (16 / 32 contiguous bytes: a warp reads 512 / 1,024
+// contiguous bytes per load) and forms sum_z pi_z L[z]; the category sum is
+// gathered by shuffles in category order, so every site lnL is the same fp64
+// value as site_root's.
+template <typename T, int C>
+__global__ void __launch_bounds__(256)
+k_root4(const T *__restrict__ L, const double *__restrict__ w, const double *__restrict__ pi,
+        const int32_t *__restrict__ cum, const double *__restrict__ pw, int p, double *__restrict__ site,
+        double *__restrict__ blocks, unsigned *__restrict__ count, double *__restrict__ out) {
+  __shared__ double red[32];
+  double part = 0.0;
+  const int lane = threadIdx.x & 31, c = lane % C;
+  const double p0 = pi[0], p1 = pi[1], p2 = pi[2], p3 = pi[3];
+  const int stride = (gridDim.x * blockDim.x) / C;
+  for (int i0 = (blockIdx.x * blockDim.x + (threadIdx.x & ~31)) / C; i0 < p; i0 += stride) {
+    const int i = i0 + lane / C;
+    const bool valid = i < p;
+    double sc = 0.0;
+    if (valid) {
+      const T *row = L + ((size_t)i * C + c) * 4;
+      sc = fma(p0, (double)row[0], sc);
+      sc = fma(p1, (double)row[1], sc);
+      sc = fma(p2, (double)row[2], sc);
+      sc = fma(p3, (double)row[3], sc);
+    }
+    double acc = 0.0;
+#pragma unroll
+    for (int k = 0; k < C; ++k) acc = fma(w[k], __shfl_sync(0xffffffffu, sc, (lane - c) + k), acc);
+    if (valid && c == 0) {
+      double l = log(acc);
+      if (cum != nullptr) l += (double)cum[i] * kLn2;
+      site[i] = l;
+      part += pw[i] * l;
+    }
+  }
+  finish_sum(part, red, blocks, count, out);
+}
+
 // ---------------------------------------------------------------------- K6
 template <typename T>
 __global__ void __launch_bounds__(256)
@@ -361,6 +433,15 @@ int launch_transition_matrices(int prec, int s, int s_pad, int c, const double *
                                                         static_cast<double *>(d_PT));
     return (int)cudaGetLastError();
   }
+  if (s == 4 && s_pad == 4) {
+    const long long th = 4LL * count * c;
+    const int blocks = (int)((th + 127) / 128);
+    if (prec == 32)
+      k_transition4<float><<<blocks, 128, 0, st>>>(c, count, d_eig, d_rates, d_idx, d_t, static_cast<float *>(d_P));
+    else
+      k_transition4<double><<<blocks, 128, 0, st>>>(c, count, d_eig, d_rates, d_idx, d_t, static_cast<double *>(d_P));
+    return (int)cudaGetLastError();
+  }
   const size_t smem = sizeof(double) * (2 * s * s + s);
   const int threads = (s <= 4) ? 32 : 256;
   for (int o = 0; o < count; o += 65535) {
@@ -394,6 +475,20 @@ int launch_root_lnl(int prec, int s, int s_pad, int c, const void *root, const d
                     double *d_site, double *d_block, unsigned *d_count, int nblocks, double *d_out,
                     void *stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (s == 4 && s_pad == 4 && (c == 1 || c == 2 || c == 4 || c == 8)) {
+#define RRL_ROOT4(T, CC)                                                                                 \
+  k_root4<T, CC><<<nblocks, 256, 0, st>>>(static_cast<const T *>(root), d_w, d_pi, cum, d_pw, p, d_site, \
+                                          d_block, d_count, d_out)
+    if (prec == 32) {
+      if (c == 1) RRL_ROOT4(float, 1); else if (c == 2) RRL_ROOT4(float, 2);
+      else if (c == 4) RRL_ROOT4(float, 4); else RRL_ROOT4(float, 8);
+    } else {
+      if (c == 1) RRL_ROOT4(double, 1); else if (c == 2) RRL_ROOT4(double, 2);
+      else if (c == 4) RRL_ROOT4(double, 4); else RRL_ROOT4(double, 8);
+    }
+#undef RRL_ROOT4
+    return (int)cudaGetLastError();
+  }
   if (prec == 32)
     k_root<float><<<nblocks, 256, 0, st>>>(static_cast<const float *>(root), s, s_pad, c, d_w, d_pi,
                                            cum, d_pw, p, p_pad, d_site, d_block, d_count, d_out);

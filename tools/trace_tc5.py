@@ -47,7 +47,7 @@ def main():
     R.rrl_update_partials(tl.inst, ops, np.array([0, b - a], np.int32))
     R.rrl_synchronize(tl.inst)
     lib = C.CDLL(LIB)
-    ev = np.zeros((16, 4096), np.int64)
+    ev = np.zeros((18, 4096), np.int64)
     kind = np.zeros(4096, np.int32)
     assert lib.rrl_debug_tc5_trace(ev.ctypes.data_as(C.c_void_p), kind.ctypes.data_as(C.c_void_p)) == 0
     ntiles = (w.p + 127) // 128
@@ -100,12 +100,15 @@ def main():
             continue
         base = ev[4, pg]
         rows.append([ev[12, g] - base, ev[13, g] - base, ev[14, g] - base, ev[15, g] - base, ev[3, g] - base,
-                     ev[4, g] - ev[3, g]])
+                     ev[4, g] - ev[3, g], ev[16, g] - base])
     if rows:
+        print("per internal phase (first 24): b_full a_full lo_full acc_empty start issue P_issued")
+        for rr in rows[:24]:
+            print("   " + " ".join(f"{x:7d}" for x in rr))
         r = np.median(np.array(rows), axis=0)
         print("MMA issuer, cycles after the previous internal phase's commit (median): "
               f"b_full {r[0]:.0f}  a_full {r[1]:.0f}  lo_full {r[2]:.0f}  acc_empty {r[3]:.0f}  start {r[4]:.0f}; "
-              f"issue {r[5]:.0f}")
+              f"issue {r[5]:.0f}; its matrix tile was issued at {r[6]:.0f}")
     tl.close()
 
 
