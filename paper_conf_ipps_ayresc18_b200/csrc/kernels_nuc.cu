@@ -63,7 +63,14 @@ constexpr int kInline = RRL_LAT_INLINE;
 // (one SM's bulk engine streams 1.3 MB while that CTA cannot retire); 2 or 4
 // inline descriptors instead of 8 0.117 / 0.118 (the pointer path for a
 // 2-operation set: 0.147); children read with ld.global.cg instead of .nc
-// (RRL_LAT_CG) 0.1174 vs 0.1173.  fp64 (tables in shared memory already) keeps 3
+// (RRL_LAT_CG) 0.1174 vs 0.1173.  The trigger position is a balance: the
+// next set's launch fires once every CTA of this one has run its prologue,
+// and the HBM round trip of the tip-state loads in that prologue paces it --
+// without those loads (timing ablation RRL_LAT_ABL=4) or with the tip states
+// prefetched into L2 the pass is slower (0.152 / 0.128 ms: the set after next
+// starts its prologue inside this set's critical section); triggering only
+// after the tip states arrived (RRL_LAT_TRIG_AFTER_TIP) 0.120, after the wait
+// 0.118, at the top 0.145.  fp64 (tables in shared memory already) keeps 3
 // CTAs per SM: at 5 it spills and is no faster.
 #ifndef RRL_LAT_MINB
 #define RRL_LAT_MINB 12
@@ -81,11 +88,15 @@ constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 #ifndef RRL_LAT_U  // items per thread on the latency path
 #define RRL_LAT_U 1
 #endif
-#ifndef RRL_LAT_ABL  // timing ablations (dev builds only; results are wrong): 1 no child exponents, 2 no rescale
+#ifndef RRL_LAT_ABL  // timing ablations (dev builds only; results are wrong): 1 no child exponents, 2 no rescale,
+                     // 4 no tip-state loads
 #define RRL_LAT_ABL 0
 #endif
 #ifndef RRL_LAT_CG  // children and their exponents read with ld.global.cg (L2 only) instead of ld.global.nc
 #define RRL_LAT_CG 0
+#endif
+#ifndef RRL_LAT_TRIG_AFTER_TIP
+#define RRL_LAT_TRIG_AFTER_TIP 0
 #endif
 #ifndef RRL_LAT_PIN
 #define RRL_LAT_PIN 0
@@ -367,8 +378,8 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
     for (int j = 0; j < U; ++j) {
       const unsigned item = (unsigned)blockIdx.x * (kLatThreads * U) + threadIdx.x + j * kLatThreads;
       const bool valid = item < nitems && (int)blockIdx.x < nchunks;
-      s1p[j] = (tip1 && valid) ? (unsigned)__ldg(S1g + item / C) : 4u;
-      s2p[j] = (tip2 && valid) ? (unsigned)__ldg(S2g + item / C) : 4u;
+      s1p[j] = (tip1 && valid) ? ((RRL_LAT_ABL & 4) ? (item / C) & 3u : (unsigned)__ldg(S1g + item / C)) : 4u;
+      s2p[j] = (tip2 && valid) ? ((RRL_LAT_ABL & 4) ? (item / C) & 3u : (unsigned)__ldg(S2g + item / C)) : 4u;
     }
   }
   if (early & 2) load_rows();
@@ -402,6 +413,16 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 #if RRL_LAT_PDL_TOP
   pdl_wait();  // everything above overlaps the previous level set
 #elif RRL_LAT_PDL_EARLY
+#if RRL_LAT_TRIG_AFTER_TIP
+  // trigger the next level set's launch only once this thread's tip states have
+  // arrived (the comparison waits on their scoreboard)
+  if (early & 1) {
+    unsigned acc = 0;
+#pragma unroll
+    for (int j = 0; j < U; ++j) acc |= s1p[j] | s2p[j];
+    if (acc == 0xffffffffu) __nanosleep(1);
+  }
+#endif
   pdl_launch();
   pdl_wait();  // everything above overlaps the previous level set
 #else
