@@ -70,7 +70,9 @@ constexpr int kInline = RRL_LAT_INLINE;
 // prefetched into L2 the pass is slower (0.152 / 0.128 ms: the set after next
 // starts its prologue inside this set's critical section); triggering only
 // after the tip states arrived (RRL_LAT_TRIG_AFTER_TIP) 0.120, after the wait
-// 0.118, at the top 0.145.  fp64 (tables in shared memory already) keeps 3
+// 0.118, at the top 0.145.  fp64 (configs[1] fp64, updatePartials): 4 / 5 /
+// 6 / 8 / 10 / 12 CTAs per SM 0.155 / 0.155 / 0.172 / 0.194 / 0.222 / 0.280
+// ms (5: one level set's 626 CTAs resident at a time); fp32 at 4-6: 0.136.  fp64 (tables in shared memory already) keeps 3
 // CTAs per SM: at 5 it spills and is no faster.
 #ifndef RRL_LAT_MINB
 #define RRL_LAT_MINB 12
@@ -111,7 +113,10 @@ constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 #define RRL_LAT_THREADS 128
 #endif
 constexpr int kLatThreads = RRL_LAT_THREADS;  // latency-path CTA size
-constexpr int kLatencyMinBlocks64 = 3 * 256 / kLatThreads;  // fp64: 768 resident threads per SM
+#ifndef RRL_LAT_MINB64
+#define RRL_LAT_MINB64 5  // fp64: 640 resident threads per SM (measured best, 4-12)
+#endif
+constexpr int kLatencyMinBlocks64 = RRL_LAT_MINB64;
 constexpr int kChunkItems = 512;  // items (pattern x category) per bulk chunk
 constexpr int kPTab = 36;         // per (branch, cat): 16 rows P[z][x] + 5 columns x 4
 
