@@ -66,7 +66,7 @@ constexpr int kInline = RRL_LAT_INLINE;
 // (RRL_LAT_CG) 0.1174 vs 0.1173.  The trigger position is a balance: the
 // next set's launch fires once every CTA of this one has run its prologue,
 // and the HBM round trip of the tip-state loads in that prologue paces it --
-// without those loads (timing ablation RRL_LAT_ABL=4) or with the tip states
+// without those loads (a timing-only build that skipped them) or with the tip states
 // prefetched into L2 the pass is slower (0.152 / 0.128 ms: the set after next
 // starts its prologue inside this set's critical section); triggering only
 // after the tip states arrived (RRL_LAT_TRIG_AFTER_TIP) 0.120, after the wait
@@ -89,10 +89,6 @@ constexpr int kLatencyMinBlocks = RRL_LAT_MINB;
 #endif
 #ifndef RRL_LAT_U  // items per thread on the latency path
 #define RRL_LAT_U 1
-#endif
-#ifndef RRL_LAT_ABL  // timing ablations (dev builds only; results are wrong): 1 no child exponents, 2 no rescale,
-                     // 4 no tip-state loads
-#define RRL_LAT_ABL 0
 #endif
 #ifndef RRL_LAT_CG  // children and their exponents read with ld.global.cg (L2 only) instead of ld.global.nc
 #define RRL_LAT_CG 0
@@ -383,8 +379,8 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
     for (int j = 0; j < U; ++j) {
       const unsigned item = (unsigned)blockIdx.x * (kLatThreads * U) + threadIdx.x + j * kLatThreads;
       const bool valid = item < nitems && (int)blockIdx.x < nchunks;
-      s1p[j] = (tip1 && valid) ? ((RRL_LAT_ABL & 4) ? (item / C) & 3u : (unsigned)__ldg(S1g + item / C)) : 4u;
-      s2p[j] = (tip2 && valid) ? ((RRL_LAT_ABL & 4) ? (item / C) & 3u : (unsigned)__ldg(S2g + item / C)) : 4u;
+      s1p[j] = (tip1 && valid) ? (unsigned)__ldg(S1g + item / C) : 4u;
+      s2p[j] = (tip2 && valid) ? (unsigned)__ldg(S2g + item / C) : 4u;
     }
   }
   if (early & 2) load_rows();
@@ -468,8 +464,8 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 #pragma unroll
         for (int z = 0; z < 4; ++z) L2[j][z] = T(0);
       }
-      ca[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum1 != nullptr) ? (RRL_LAT_CG ? __ldcg(op.cum1 + pat) : __ldg(op.cum1 + pat)) : 0;
-      cb[j] = (!(RRL_LAT_ABL & 1) && scale_w && valid && cat == 0 && op.cum2 != nullptr) ? (RRL_LAT_CG ? __ldcg(op.cum2 + pat) : __ldg(op.cum2 + pat)) : 0;
+      ca[j] = (scale_w && valid && cat == 0 && op.cum1 != nullptr) ? (RRL_LAT_CG ? __ldcg(op.cum1 + pat) : __ldg(op.cum1 + pat)) : 0;
+      cb[j] = (scale_w && valid && cat == 0 && op.cum2 != nullptr) ? (RRL_LAT_CG ? __ldcg(op.cum2 + pat) : __ldg(op.cum2 + pat)) : 0;
     }
     if constexpr (!kRegP) {
       if (!tables) {  // block-uniform, first chunk only
@@ -496,11 +492,7 @@ k_partials_nuc(const __grid_constant__ OpPack pack, int p, int nchunks, int earl
 #ifdef RRL_LAT_TRACE
       if (j == 0 && threadIdx.x == 0 && t_ld == 0) t_ld = gtime_after((float)r[0] + (float)ca[0] + (float)cb[0]);
 #endif
-#if RRL_LAT_ABL & 2  // ablation (timing experiments only): plain store, no rescale
-      if (valid) V4<T>::st(out + (size_t)item * 4, r);
-#else
       finish_item<T, C>(op, r, valid, pat, cat, ca[j], cb[j], out + (size_t)item * 4);
-#endif
     }
   }
 #ifdef RRL_LAT_TRACE
