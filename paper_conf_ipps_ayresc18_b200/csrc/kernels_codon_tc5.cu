@@ -98,7 +98,10 @@ constexpr int kThr = 15 * 32;
 // slot (RRL_TC5_NB=3, the MMA issuer's longest wait was its P tile) -> 1.431.
 // No gain: the lo hand-over per K-half (RRL_TC5_LOSPLIT, 1.550 / 1.530 with
 // smem / TMEM lo), two TMEM lo slots with the last category kept in registers
-// (RRL_TC5_NLO=2, 1.475-1.518), tip columns from P^T (RRL_TC5_TIP_PT, 1.734).
+// (RRL_TC5_NLO=2, 1.475-1.518), tip columns from P^T (RRL_TC5_TIP_PT, 1.734),
+// a fourth matrix slot instead of the third child tile (1.442), tip phases'
+// P tiles released per epilogue warp instead of behind a 256-thread barrier
+// (1.4315 vs 1.4321, backed out).
 // RRL_TC5_LOSPLIT=1: the lo tile is handed over per K-half (two full / empty
 // barrier pairs per lo slot): the MMAs of K-half 0 start once the converters
 // finished that half, and the converters start the next phase's K-half 0 as
