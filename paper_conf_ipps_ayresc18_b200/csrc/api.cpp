@@ -90,6 +90,14 @@ struct Instance {
   cudaGraphExec_t graph = nullptr;       // replay of the set launches
   cudaStream_t graph_stream = nullptr;
   int graph_kernels = 0;
+  // K1 deferred into the level-set graph (RRL_FLAG_CUDA_GRAPH, profiling off):
+  // rrl_update_transition_matrices records it, the next rrl_update_partials
+  // replays it as the graph's first node; any other call launches it first.
+  bool k1_pending = false;
+  int k1_eig = 0, k1_count = 0;
+  bool graph_has_k1 = false;               // the captured graph starts with K1 for:
+  int graph_k1_eig = -1, graph_k1_count = -1;
+  const double *graph_k1_t = nullptr;
 
   bool profiling = false;
   std::vector<EvPair> events;
@@ -133,11 +141,25 @@ int use_device(Instance *I) {
   return 0;
 }
 
-#define GET(I, id)                                                                  \
+int launch_k1(Instance *I, int eigen_idx, int count);
+// A deferred K1 goes onto the stream before anything else the instance does.
+int flush_k1(Instance *I) {
+  if (!I->k1_pending) return 0;
+  I->k1_pending = false;
+  return launch_k1(I, I->k1_eig, I->k1_count);
+}
+
+#define GET_RAW(I, id)                                                              \
   Instance *I = get(id);                                                            \
   if (!I) return fail(RRL_ERROR_UNINITIALIZED_INSTANCE, "no such instance");        \
   {                                                                                 \
     int r_ = use_device(I);                                                         \
+    if (r_ < 0) return r_;                                                          \
+  }
+#define GET(I, id)                                                                  \
+  GET_RAW(I, id)                                                                    \
+  {                                                                                 \
+    int r_ = flush_k1(I);                                                           \
     if (r_ < 0) return r_;                                                          \
   }
 
@@ -193,6 +215,20 @@ int drop_graphs(Instance *I) {
   if (I->graph) cudaGraphExecDestroy(I->graph);
   I->graph = nullptr;
   return 0;
+}
+
+// K1 on the instance stream (eagerly, or inside the level-set graph's capture).
+int launch_k1(Instance *I, int eigen_idx, int count) {
+  const size_t eig_sz = 2 * (size_t)I->s * I->s + I->s;
+  {
+    Timed tm(I, 1);
+    CKL(launch_transition_matrices(I->prec, I->s, I->s_pad, I->c, I->d_eig + eig_sz * eigen_idx,
+                                   I->d_rates + (size_t)eigen_idx * I->c, I->d_midx, I->d_t, count, I->d_P,
+                                   I->d_Plo, I->d_PT, I->stream));
+  }
+  I->prof.matrices_launches += (count + 65534) / 65535;
+  I->prof.kernel_launches += (count + 65534) / 65535;
+  return RRL_SUCCESS;
 }
 
 void destroy(Instance *I) {
@@ -631,17 +667,16 @@ int rrl_update_transition_matrices(int inst, int eigen_idx, const int32_t *matri
                        I->stream));
     I->t_count = count;
   }
-  const size_t eig_sz = 2 * (size_t)I->s * I->s + I->s;
-  {
-    Timed tm(I, 1);
-    CKL(launch_transition_matrices(I->prec, I->s, I->s_pad, I->c, I->d_eig + eig_sz * eigen_idx,
-                                   I->d_rates + (size_t)eigen_idx * I->c, I->d_midx, I->d_t, count, I->d_P,
-                                   I->d_Plo, I->d_PT, I->stream));
+  if ((I->flags & RRL_FLAG_CUDA_GRAPH) && I->stream != nullptr && !I->profiling) {
+    // deferred: the next level-set graph replays it as its first node
+    I->k1_pending = true;
+    I->k1_eig = eigen_idx;
+    I->k1_count = count;
+    return RRL_SUCCESS;
   }
-  I->prof.matrices_launches += (count + 65534) / 65535;
-  I->prof.kernel_launches += (count + 65534) / 65535;
-  return RRL_SUCCESS;
+  return launch_k1(I, eigen_idx, count);
 }
+
 
 int rrl_set_transition_matrix(int inst, int idx, const double *P) {
   GET(I, inst);
@@ -692,7 +727,7 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
 
 int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t *set_offsets,
                         int set_count) {
-  GET(I, inst);
+  GET_RAW(I, inst);  // a deferred K1 becomes the first node of the level-set graph
   return update_partials_impl(I, ops, nullptr, op_count, set_offsets, set_count);
 }
 
@@ -982,15 +1017,31 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
 
   // (the legacy default stream cannot be captured: eager launches there)
   const bool use_graph = (I->flags & RRL_FLAG_CUDA_GRAPH) && I->stream != nullptr;
+  const bool with_k1 = use_graph && I->k1_pending && !I->profiling;
+  if (!with_k1) {
+    int r = flush_k1(I);
+    if (r < 0) return r;
+  }
   if (use_graph) {
-    if (I->graph && I->graph_stream != I->stream) {
+    if (I->graph && (I->graph_stream != I->stream || I->graph_has_k1 != with_k1 ||
+                     (with_k1 && (I->graph_k1_eig != I->k1_eig || I->graph_k1_count != I->k1_count ||
+                                  I->graph_k1_t != I->d_t)))) {
       int r = drop_graphs(I);
       if (r < 0) return r;
     }
     if (!I->graph) {
       cudaGraph_t g;
       CK(cudaStreamBeginCapture(I->stream, cudaStreamCaptureModeThreadLocal));
-      int e = launch_all(true);
+      int e = 0;
+      if (with_k1) {  // K1 as the graph's first node (set 0 already waits for its predecessor)
+        e = launch_transition_matrices(I->prec, I->s, I->s_pad, I->c,
+                                       I->d_eig + (2 * (size_t)I->s * I->s + I->s) * I->k1_eig,
+                                       I->d_rates + (size_t)I->k1_eig * I->c, I->d_midx, I->d_t, I->k1_count,
+                                       I->d_P, I->d_Plo, I->d_PT, I->stream);
+        if (e != 0) e = fail(RRL_ERROR_CUDA, std::string("K1 capture: ") +
+                                                 cudaGetErrorString(static_cast<cudaError_t>(e)));
+      }
+      if (e == 0) e = launch_all(true);
       cudaError_t ce = cudaStreamEndCapture(I->stream, &g);
       if (e < 0) return e;
       CK(ce);
@@ -999,6 +1050,15 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       CK(ie);
       I->graph_stream = I->stream;
       I->graph_kernels = kl;
+      I->graph_has_k1 = with_k1;
+      I->graph_k1_eig = with_k1 ? I->k1_eig : -1;
+      I->graph_k1_count = with_k1 ? I->k1_count : -1;
+      I->graph_k1_t = with_k1 ? I->d_t : nullptr;
+    }
+    if (with_k1) {  // replayed inside the graph
+      I->k1_pending = false;
+      I->prof.matrices_launches += (I->k1_count + 65534) / 65535;
+      I->prof.kernel_launches += (I->k1_count + 65534) / 65535;
     }
     {
       // profiling: one event pair around the whole replay on the launching
