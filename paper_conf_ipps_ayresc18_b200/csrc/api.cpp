@@ -95,6 +95,16 @@ struct Instance {
   // replays it as the graph's first node; any other call launches it first.
   bool k1_pending = false;
   int k1_eig = 0, k1_count = 0;
+  // The level-set graph's launch deferred to the next call (graph mode,
+  // profiling off): rrl_calculate_root_log_likelihoods_device replays it and
+  // K4 as one graph (child graph + K4 node), any other call launches it first.
+  bool pass_pending = false;
+  cudaGraph_t graph_tmpl = nullptr;        // the captured level-set graph (child of root_graph)
+  unsigned graph_gen = 0;                  // bumped at every (re)capture
+  cudaGraphExec_t root_graph = nullptr;    // [level-set graph] -> K4
+  unsigned root_gen = ~0u;
+  int root_key[4] = {-2, -2, -2, -2};
+  double *root_out = nullptr;
   bool graph_has_k1 = false;               // the captured graph starts with K1 for:
   int graph_k1_eig = -1, graph_k1_count = -1;
   const double *graph_k1_t = nullptr;
@@ -142,9 +152,12 @@ int use_device(Instance *I) {
 }
 
 int launch_k1(Instance *I, int eigen_idx, int count);
-// A deferred K1 goes onto the stream before anything else the instance does.
+int flush_pass(Instance *I);
+// A deferred K1 (and a deferred level-set graph) go onto the stream before
+// anything else the instance does.
 int flush_k1(Instance *I) {
-  if (!I->k1_pending) return 0;
+  int r = flush_pass(I);
+  if (r < 0 || !I->k1_pending) return r;
   I->k1_pending = false;
   return launch_k1(I, I->k1_eig, I->k1_count);
 }
@@ -214,6 +227,19 @@ void drain_events(Instance *I) {
 int drop_graphs(Instance *I) {
   if (I->graph) cudaGraphExecDestroy(I->graph);
   I->graph = nullptr;
+  if (I->graph_tmpl) cudaGraphDestroy(I->graph_tmpl);
+  I->graph_tmpl = nullptr;
+  if (I->root_graph) cudaGraphExecDestroy(I->root_graph);
+  I->root_graph = nullptr;
+  I->graph_gen += 1;
+  return 0;
+}
+
+int flush_pass(Instance *I) {
+  if (!I->pass_pending) return 0;
+  I->pass_pending = false;
+  Timed tm(I, 0);
+  CK(cudaGraphLaunch(I->graph, I->stream));
   return 0;
 }
 
@@ -234,7 +260,7 @@ int launch_k1(Instance *I, int eigen_idx, int count) {
 void destroy(Instance *I) {
   cudaSetDevice(I->device);
   if (I->stream) cudaStreamSynchronize(I->stream);
-  if (I->graph) cudaGraphExecDestroy(I->graph);
+  drop_graphs(I);
   for (void *t : I->tip_partials)
     if (t) cudaFree(t);
   void *ptrs[] = {I->d_partials, I->d_states, I->d_P,    I->d_scale, I->d_eig,  I->d_rates,
@@ -728,6 +754,10 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
 int rrl_update_partials(int inst, const rrl_op *ops, int op_count, const int32_t *set_offsets,
                         int set_count) {
   GET_RAW(I, inst);  // a deferred K1 becomes the first node of the level-set graph
+  {
+    int r = flush_pass(I);  // a previous deferred pass runs first
+    if (r < 0) return r;
+  }
   return update_partials_impl(I, ops, nullptr, op_count, set_offsets, set_count);
 }
 
@@ -1046,8 +1076,9 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       if (e < 0) return e;
       CK(ce);
       cudaError_t ie = cudaGraphInstantiate(&I->graph, g, 0);
-      cudaGraphDestroy(g);
+      if (ie != cudaSuccess) cudaGraphDestroy(g);
       CK(ie);
+      I->graph_tmpl = g;  // kept: the child of the [level sets -> K4] graph
       I->graph_stream = I->stream;
       I->graph_kernels = kl;
       I->graph_has_k1 = with_k1;
@@ -1060,7 +1091,9 @@ static int update_partials_impl(Instance *I, const rrl_op *ops, const int32_t *r
       I->prof.matrices_launches += (I->k1_count + 65534) / 65535;
       I->prof.kernel_launches += (I->k1_count + 65534) / 65535;
     }
-    {
+    if (!I->profiling) {
+      I->pass_pending = true;  // launched by the next call (with K4 by the device root call)
+    } else {
       // profiling: one event pair around the whole replay on the launching
       // stream; per-launch duration = region time / launches (events inside
       // the graph would break the programmatic-dependent-launch overlap).
@@ -1163,9 +1196,47 @@ int rrl_calculate_root_log_likelihoods(int inst, int root_buffer, int cat_weight
 
 int rrl_calculate_root_log_likelihoods_device(int inst, int root_buffer, int cat_weights_idx,
                                               int freqs_idx, int cumulative_idx, double *d_out) {
-  GET(I, inst);
+  GET_RAW(I, inst);
   if (!d_out) return fail(RRL_ERROR_GENERAL, "d_out NULL");
-  return root_common(I, root_buffer, cat_weights_idx, freqs_idx, cumulative_idx, d_out);
+  if (!I->pass_pending || I->profiling || !I->graph_tmpl) {
+    int r = flush_k1(I);
+    if (r < 0) return r;
+    return root_common(I, root_buffer, cat_weights_idx, freqs_idx, cumulative_idx, d_out);
+  }
+  // the deferred level-set graph and K4 as one graph
+  const int key[4] = {root_buffer, cat_weights_idx, freqs_idx, cumulative_idx};
+  if (!I->root_graph || I->root_gen != I->graph_gen || I->root_out != d_out ||
+      std::memcmp(key, I->root_key, sizeof(key)) != 0) {
+    if (I->root_graph) cudaGraphExecDestroy(I->root_graph);
+    I->root_graph = nullptr;
+    cudaGraph_t k4g = nullptr;
+    CK(cudaStreamBeginCapture(I->stream, cudaStreamCaptureModeThreadLocal));
+    const int r = root_common(I, root_buffer, cat_weights_idx, freqs_idx, cumulative_idx, d_out);
+    const cudaError_t ce = cudaStreamEndCapture(I->stream, &k4g);
+    if (r < 0) {
+      if (k4g) cudaGraphDestroy(k4g);
+      return r;
+    }
+    CK(ce);
+    cudaGraph_t g = nullptr;
+    cudaGraphNode_t pass = nullptr, k4 = nullptr;
+    cudaError_t e = cudaGraphCreate(&g, 0);
+    if (e == cudaSuccess) e = cudaGraphAddChildGraphNode(&pass, g, nullptr, 0, I->graph_tmpl);
+    if (e == cudaSuccess) e = cudaGraphAddChildGraphNode(&k4, g, &pass, 1, k4g);
+    if (e == cudaSuccess) e = cudaGraphInstantiate(&I->root_graph, g, 0);
+    if (g) cudaGraphDestroy(g);
+    cudaGraphDestroy(k4g);
+    CK(e);
+    I->root_gen = I->graph_gen;
+    I->root_out = d_out;
+    std::memcpy(I->root_key, key, sizeof(key));
+  } else {
+    I->prof.root_launches += 1;  // (root_common counted the captured launch)
+    I->prof.kernel_launches += 1;
+  }
+  I->pass_pending = false;
+  CK(cudaGraphLaunch(I->root_graph, I->stream));
+  return RRL_SUCCESS;
 }
 
 int rrl_calculate_edge_log_likelihoods(int inst, int parent_buffer, int child_buffer, int matrix_idx,
